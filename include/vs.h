@@ -1,0 +1,197 @@
+/* include/vs.h -- C ABI of the B200-native virtual-screening hot path.
+ *
+ * What it computes (PAPER.md = Imbernon, Cecilia, Gimenez, PMAM'16;
+ * "P:N" = line N of PAPER.md; "Rn" = reading n in DESIGN.md §3):
+ *   - the scoring function of a rigid ligand pose placed near a receptor
+ *     spot: a sum over all ligand-atom x receptor-atom pairs of
+ *     electrostatic, Lennard-Jones and hydrogen-bond terms
+ *     ("computations between pairs of atoms in the protein and the
+ *     ligand"; P:55 Coulomb + Lennard-Jones; P:84 spots, conformations;
+ *     pair terms R1-R8);
+ *   - the metaheuristic of Algorithm 1 (Initialize, End, Select,
+ *     Combine, Improve, Include) run independently at every spot (P:84,
+ *     P:140), with the Table 4 parameters as presets.
+ *
+ * Conventions (all functions):
+ *   - extern "C", never throw, never abort; a non-OK status leaves a
+ *     thread-local message readable with vs_last_error().
+ *   - The caller owns every buffer it passes.  vs_create deep-copies its
+ *     inputs; outputs go to caller-sized buffers; on error the output
+ *     buffers are unspecified and vs_create returns *out = NULL.
+ *   - A ctx is bound to one CUDA device and used by one host thread at a
+ *     time; several ctx may share a device.
+ *   - After VS_ERR_CUDA a ctx is poisoned: every later call except
+ *     vs_destroy returns VS_ERR_CUDA.
+ *   - Units: Angstrom, elementary charge, kcal/mol.  Arrays are row-major
+ *     fp32 / int32 host arrays unless a name starts with d_ (device memory
+ *     of the ctx's device).
+ */
+#ifndef VS_H
+#define VS_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define VS_ABI_VERSION 1
+
+typedef struct vs_ctx vs_ctx; /* opaque; owned by the library */
+
+typedef enum {
+  VS_OK = 0,
+  VS_ERR_INVALID_ARGUMENT = 1,   /* NULL pointer, bad count, bad type id, non-finite input */
+  VS_ERR_POSE_OUT_OF_REGION = 2, /* cutoff mode: |t_k| > region_half_width (R10) */
+  VS_ERR_ZERO_QUATERNION = 3,    /* quaternion with zero norm */
+  VS_ERR_CUDA = 4,               /* CUDA runtime failure (ctx poisoned) */
+  VS_ERR_OUT_OF_MEMORY = 5,      /* host or device allocation failed */
+  VS_ERR_UNSUPPORTED = 6         /* valid request this build does not implement */
+} vs_status;
+
+/* Scoring-function parameters.  vs_score_params_default() fills:
+ *   coulomb_k 332.0636 (R2), dielectric 0 = eps(r) = 4r (R3), eps_r 1,
+ *   cutoff 12 A with electrostatic shift (1 - r^2/rc^2)^2 (R6),
+ *   region_half_width 3 A (R10), hb_eps 5 kcal/mol, hb_r0 1.9 A (R5),
+ *   r2_min 0.01 A^2 (R7), n_types 0 = built-in 7-type table:
+ *     id: 0 C, 1 N, 2 O, 3 S, 4 H, 5 HD (polar H), 6 X (dummy)
+ *     sigma 3.400 3.250 2.960 3.564 2.650 1.069 0
+ *     eps   0.1094 0.170 0.210 0.250 0.0157 0.0157 0
+ *     role  -  acc  acc  -  -  donor  -       (1 donor, 2 acceptor)
+ * cutoff <= 0 or +inf selects all-pairs mode (the paper's brute-force
+ * reading); a finite cutoff selects per-spot binned lists, exact for
+ * every pose inside the region (R10).  dielectric 1 (constant eps_r,
+ * E = k qi qj / (eps_r r)) is accepted. */
+typedef struct {
+  float coulomb_k;
+  int dielectric;
+  float eps_r;
+  float cutoff;
+  float region_half_width;
+  float hb_eps, hb_r0;
+  float r2_min;
+  int n_types;                /* 0 -> built-in table; else 1..64 entries below */
+  const float* type_sigma;    /* [n_types] A   (>= 0) */
+  const float* type_eps;      /* [n_types] kcal/mol (>= 0) */
+  const int* type_hb_role;    /* [n_types] 0 none, 1 donor, 2 acceptor */
+} vs_score_params;
+
+/* Metaheuristic parameters (Algorithm 1; Table 4).
+ * population P (1..2048; >= 2 when generations > 0), generations G >= 0
+ * (End condition, R20), ls_steps L >= 0 (Improve, R16), improve_frac f in
+ * [0,1] (Table 4 "% of elements to be improved"; m = clamp(round(f*P),1,P)
+ * elements, R17), p_mut in [0,1] (R15), step sizes >= 0 (A, radians-ish
+ * quaternion increments). */
+typedef struct {
+  int population, generations, ls_steps;
+  float improve_frac, p_mut, mut_trans, mut_rot, ls_trans, ls_rot;
+} vs_mh_params;
+
+void vs_score_params_default(vs_score_params* out);
+
+/* m = 1..4 -> M1..M4 of Table 4:
+ *   M1 GA: P 64, f 0;  M2: P 64, f 1, L 8;  M3: P 64, f 0.2, L 8;
+ *   M4: P 1024, G 0, f 1, L 8 ("only one step").
+ *   G = 50 for M1-M3 (the paper does not report it, R22); p_mut 0.1,
+ *   mut 1.0 A / 0.25, ls 0.5 A / 0.10.
+ * Returns VS_ERR_INVALID_ARGUMENT for another m or out == NULL. */
+vs_status vs_mh_preset(int m, vs_mh_params* out);
+
+/* Builds a scoring context on CUDA device `cuda_device`.
+ *   rec_xyz [n_rec][3], rec_q [n_rec], rec_type [n_rec]  receptor atoms
+ *   lig_xyz [n_lig][3], lig_q [n_lig], lig_type [n_lig]  ligand atoms, 1 <= n_lig <= 256
+ *   spot_xyz [n_spots][3]                                spot centres (R9)
+ *   sp: NULL -> defaults.
+ * The ligand is centred on its centroid (fp64 sum, rounded to fp32 once;
+ * l_i = lig_xyz_i - centroid in fp32, R11).  In cutoff mode the per-spot
+ * receptor lists (atoms within T*sqrt(3) + max|l_i| + rc + 0.01 A of the
+ * spot centre, R10) are built on the device here.
+ * Errors: VS_ERR_INVALID_ARGUMENT (NULL / counts / type ids / non-finite /
+ * bad params), VS_ERR_CUDA, VS_ERR_OUT_OF_MEMORY.  *out = NULL on error. */
+vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec_type, int32_t n_rec,
+                    const float* lig_xyz, const float* lig_q, const int32_t* lig_type, int32_t n_lig,
+                    const float* spot_xyz, int32_t n_spots, const vs_score_params* sp, int32_t cuda_device,
+                    vs_ctx** out);
+
+/* Scores n poses (host buffers; synchronous).
+ *   spot [n]         spot id of each pose (0 <= id < n_spots)
+ *   quat_wxyz [n][4] rotation quaternion (w,x,y,z); need not be unit (R11), must be non-zero
+ *   trans [n][3]     translation of the ligand centroid relative to the spot centre
+ *   score_out [n]    score in kcal/mol (fp32)
+ * x_i = c_spot + t + R(q) l_i;  score = sum_i sum_j e(i, j).
+ * n == 0 is a no-op.  Errors: VS_ERR_INVALID_ARGUMENT (NULL, n < 0, bad
+ * spot id, non-finite), VS_ERR_ZERO_QUATERNION, VS_ERR_POSE_OUT_OF_REGION
+ * (cutoff mode only), VS_ERR_CUDA. */
+vs_status vs_score_poses(vs_ctx* c, int64_t n, const int32_t* spot, const float* quat_wxyz, const float* trans,
+                         float* score_out);
+
+/* Same on device buffers, asynchronous on `cuda_stream` (a cudaStream_t;
+ * NULL = legacy default stream).  Poses that fail validation get a NaN
+ * score instead of an error status (no host round trip). */
+vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_quat,
+                                const float* d_trans, float* d_score, void* cuda_stream);
+
+/* Runs the metaheuristic independently at n_sel spots (synchronous).
+ *   spot_ids [n_sel] global spot ids (NULL -> all spots, n_sel must be 0 or
+ *            n_spots); the id keys the Philox streams (R23), so a spot's
+ *            result does not depend on which call / GPU / chunk ran it.
+ *   best_pose_out [n_sel][7] = (w,x,y,z,tx,ty,tz) of the best individual
+ *   best_score_out [n_sel]   its score (fp32, kcal/mol)
+ * Errors: VS_ERR_INVALID_ARGUMENT (params, ids), VS_ERR_CUDA, VS_ERR_OUT_OF_MEMORY. */
+vs_status vs_run(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                 float* best_pose_out, float* best_score_out);
+
+/* Same, asynchronous on `cuda_stream`; outputs in device memory.  spot_ids
+ * is a HOST array (validated on the host).  The ctx's workspace is reused:
+ * do not overlap two vs_run_async calls of one ctx on different streams. */
+vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                       float* d_best_pose, float* d_best_score, void* cuda_stream);
+
+void vs_destroy(vs_ctx* c); /* NULL-safe; synchronises the ctx's device work */
+const char* vs_last_error(void);
+int vs_abi_version(void);
+
+/* ---- instrumentation ---------------------------------------------------- */
+typedef struct {
+  uint64_t kernel_launches;  /* all kernels this ctx launched */
+  uint64_t score_launches;   /* scoring-kernel launches (plain + fused local search) */
+  uint64_t poses_scored;     /* poses scored (incl. local-search proposals) */
+  uint64_t pairs;            /* algorithmic atom pairs: n_lig x list length per scored pose */
+  double score_ms;           /* summed CUDA-event time of scoring launches (timing enabled) */
+  uint64_t timed_launches;   /* launches covered by score_ms */
+} vs_stats;
+
+/* enable = 1: bracket every scoring launch with CUDA events on its stream. */
+vs_status vs_set_timing(vs_ctx* c, int enable);
+/* Synchronises the ctx's device and returns counters since the last reset. */
+vs_status vs_get_stats(vs_ctx* c, vs_stats* out);
+vs_status vs_reset_stats(vs_ctx* c);
+/* Per-spot receptor list lengths (cutoff mode) or n_rec (all pairs). */
+vs_status vs_list_lengths(vs_ctx* c, int32_t* out /*[n_spots]*/);
+
+/* ---- debug / lockstep trace -------------------------------------------- */
+typedef enum {
+  VS_TRACE_INIT = 0,      /* S after Initialize's generation, before scoring (score field 0) */
+  VS_TRACE_SCORED = 1,    /* population after scoring (S at g = 0, Scom at g >= 1) */
+  VS_TRACE_SELECT = 2,    /* J: indices of the elements Improve works on (idx only) */
+  VS_TRACE_LS = 3,        /* population after local-search step l */
+  VS_TRACE_SORTED = 4,    /* S after the generation-0 sort */
+  VS_TRACE_COMBINED = 5,  /* Scom after Select + Combine, before scoring */
+  VS_TRACE_INCLUDED = 6   /* S after Include at generation g */
+} vs_trace_stage;
+
+/* poses8 [n_sel][count][8] = (w,x,y,z,tx,ty,tz,score) or NULL;
+ * idx [n_sel][count] or NULL.  Host memory valid during the call only. */
+typedef void (*vs_trace_fn)(void* user, int32_t stage, int32_t g, int32_t l, int32_t n_sel, int32_t count,
+                            const float* poses8, const int32_t* idx);
+
+/* vs_run with a callback after every stage (synchronises at each stage). */
+vs_status vs_run_trace(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                       float* best_pose_out, float* best_score_out, vs_trace_fn fn, void* user);
+
+/* Device Philox4x32-10 for n counters: ctr [n][4], key [2] -> out [n][4]
+ * (host buffers; for known-answer tests of the device generator). */
+vs_status vs_debug_philox(int64_t n, const uint32_t* ctr, const uint32_t* key, uint32_t* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* VS_H */
