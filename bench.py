@@ -1,0 +1,376 @@
+#!/usr/bin/env python
+"""Benchmark of the virtual-screening hot path (one JSON line on rank 0).
+
+A step = one full metaheuristic run (Algorithm 1, preset
+M3 of Table 4 P:232-237 with the config's population / generations) over
+every spot of the configured synthetic workload: pose generation, scoring of
+every individual and local-search proposal, selection, on device.
+
+  python bench.py [--gpus N --steps K --warmup W] [--config medium] [--preset 3]
+  torchrun --nproc-per-node N bench.py --gpus N ...        (one process per GPU, NCCL)
+  python bench.py --impl reference ...                      (the fp64 CPU oracle arm)
+
+metric: atom-pair interactions/s (BASELINE.json); a pair = one ligand atom x
+one receptor atom of the spot's streamed list (n_lig x list length per pose;
+SURVEY.md §8(d)).  Poses/s are reported alongside.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "atom-pair interactions/s and scored poses/s at 1/2/4/8 B200; % FP32 roofline"
+N_SM = 148
+LANES = 128
+OPS_CUTOFF, OPS_ALLPAIRS = 25, 20   # canonical issue slots per pair
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="medium")
+    ap.add_argument("--preset", type=int, default=3)
+    ap.add_argument("--generations", type=int, default=None, help="override the config's G")
+    ap.add_argument("--mode", choices=["cutoff", "allpairs"], default="cutoff")
+    ap.add_argument("--scaling", choices=["weak", "strong"], default="weak")
+    ap.add_argument("--seed", type=int, default=42)
+    ap.add_argument("--e2e-steps", type=int, default=None)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-clocks", action="store_true")
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region (B200_PROFILING.md)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int, enabled: bool = True):
+        self.idx = gpu_index
+        self.proc = None
+        self.lines: list[str] = []
+        self.enabled = enabled
+
+    def start(self):
+        if not self.enabled:
+            return
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "100", "-i", str(self.idx)],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self) -> dict | None:
+        if not self.proc:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = max(mx, float(f[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except (OSError, ValueError):
+        return {}
+
+
+def ncu_traffic(config: str):
+    """Per-launch DRAM bytes of the scoring kernel from the committed ncu --set full summary."""
+    import glob
+    for f in sorted(glob.glob(os.path.join(ROOT, "profiles", "*ncu_summary*.json")), reverse=True):
+        try:
+            d = json.load(open(f))
+            v = d.get("score_kernel", {}).get(config, {}).get("dram_bytes_per_launch")
+            if v is not None:
+                return v
+        except (OSError, ValueError):
+            pass
+    return None
+
+
+# ---------------------------------------------------------------- oracle arm / cpu baseline
+def oracle_sample(prob, sp_kw, mp_kw, list_len, seed, n_spots_sample: int, generations: int):
+    """Time the fp64 oracle (as it stands) on a bounded sample of the workload.
+
+    Returns (seconds, workload pairs in the sample, poses in the sample, threads)."""
+    import oracle
+    o = oracle.Oracle.from_problem(prob, oracle.score_params(**sp_kw))
+    mp = oracle.mh_preset(mp_kw["preset"], population=mp_kw["population"], generations=generations)
+    ids = np.arange(n_spots_sample, dtype=np.int32)
+    t0 = time.perf_counter()
+    o.run(mp, seed, ids)
+    dt = time.perf_counter() - t0
+    poses = o.pairs_evaluated() // (prob.cfg.n_lig * prob.cfg.n_rec)
+    per_spot = poses // n_spots_sample
+    pairs = int(sum(int(list_len[s]) for s in ids)) * prob.cfg.n_lig * per_spot
+    return dt, pairs, poses, oracle.get_threads()
+
+
+def list_lengths_host(prob, cutoff: float, T: float = 3.0):
+    """Per-spot list lengths as the library defines them (reach = T sqrt3 + max|l| + rc + 0.01)."""
+    if not cutoff > 0:
+        return np.full(len(prob.spots), prob.cfg.n_rec, np.int64)
+    lig = prob.lig.xyz.astype(np.float64)
+    cen = np.float32(lig.mean(0))
+    rmax = np.linalg.norm((prob.lig.xyz - cen).astype(np.float64), axis=1).max()
+    reach = T * np.sqrt(3) + rmax + cutoff + 0.01
+    out = []
+    rec = prob.rec.xyz.astype(np.float32)
+    for c in prob.spots:
+        d = rec - c
+        out.append(int(((d * d).sum(1) <= np.float32(reach * reach)).sum()))
+    return np.array(out)
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle on the host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    from paper_conf_ppopp_imbernoncg16_b200 import synth
+    prob = synth.make_problem(args.config)
+    cutoff = 12.0 if args.mode == "cutoff" else 0.0
+    lens = list_lengths_host(prob, cutoff)
+    P = prob.cfg.population
+    n_s, G = 1, 2 if args.config in ("medium", "large", "sweep") else min(prob.cfg.generations, 5)
+    mp_kw = {"preset": args.preset, "population": P}
+    times, pairs, poses, cores = [], 0, 0, 1
+    for i in range(args.warmup + args.steps):
+        dt, pr, po, cores = oracle_sample(prob, {"cutoff": cutoff}, mp_kw, lens, args.seed, n_s, G)
+        if i >= args.warmup:
+            times.append(dt)
+            pairs, poses = pr, po
+    ms = 1e3 * statistics.mean(times)
+    val = pairs / (ms * 1e-3)
+    sample = f"oracle vso_run on {n_s} spot(s) x {G} generations (P={P}, preset M{args.preset}) of {args.config}"
+    print(json.dumps({
+        "metric": METRIC, "value": val, "unit": "pairs/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": args.scaling,
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+        "config": {"workload": args.config, "preset": f"M{args.preset}", "mode": args.mode, "sample": sample},
+        "poses_per_s": poses / (ms * 1e-3),
+        "cpu_baseline": {"value": val, "unit": "pairs/s", "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": val, "unit": "pairs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+# ---------------------------------------------------------------- our arm
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ppopp_imbernoncg16_b200 import dist as vdist
+    from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    prob = synth.make_problem(args.config)
+    cfg = prob.cfg
+    G = cfg.generations if args.generations is None else args.generations
+    cutoff = 12.0 if args.mode == "cutoff" else 0.0
+    sp = vs.score_params(cutoff=cutoff)
+    mp = vs.mh_preset(args.preset, population=cfg.population, generations=G)
+    ctx = vs.Context.from_problem(prob, sp, device=local)
+    n_spots = cfg.n_spots
+    stream = torch.cuda.Stream(device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # > 126 MB L2
+    best_pose = torch.empty((n_spots, 7), dtype=torch.float32, device=dev)
+    best_score = torch.empty(n_spots, dtype=torch.float32, device=dev)
+    schedule = vdist.chunk_schedule(n_spots, world, min_chunk=4) if args.scaling == "strong" else None
+    store = dist.distributed_c10d._get_default_store() if world > 1 else None
+
+    def step(i: int):
+        """One whole-job pass: returns this rank's records (device tensor) for the gather."""
+        with torch.cuda.stream(stream):
+            flush.zero_()
+            if args.scaling == "weak":
+                ctx.run_async(mp, args.seed + rank, None, best_pose, best_score, stream)
+                ids = torch.arange(n_spots, dtype=torch.float32, device=dev)
+                rec = torch.cat([ids[:, None], best_score[:, None], best_pose], 1)
+            else:
+                parts = []
+
+                def work(a, b):
+                    ctx.run_async(mp, args.seed, np.arange(a, b, dtype=np.int32), best_pose[a:b], best_score[a:b],
+                                  stream)
+                    ids = torch.arange(a, b, dtype=torch.float32, device=dev)
+                    parts.append(torch.cat([ids[:, None], best_score[a:b, None], best_pose[a:b]], 1))
+
+                if world > 1:
+                    vdist.claim_chunks(store, f"q{i}", schedule, work)
+                else:
+                    for a, b in schedule:
+                        work(a, b)
+                rec = torch.cat(parts) if parts else torch.zeros((0, vdist.REC), device=dev)
+            if world > 1:
+                vdist.gather_records(rec, dev)
+        return rec
+
+    for i in range(args.warmup):
+        step(-1 - i)
+    torch.cuda.synchronize(dev)
+    ctx.reset_stats()
+    ctx.set_timing(True)
+    clocks = ClockSampler(local, enabled=(rank == 0 and not args.no_clocks))
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for i in range(args.steps):
+        step(i)
+    e1.record(stream)
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms_rank = e0.elapsed_time(e1)
+    st = ctx.stats()
+    ctx.set_timing(False)
+    # whole-job totals and max-over-ranks time
+    tot = torch.tensor([st["pairs"], st["poses_scored"], st["kernel_launches"]], dtype=torch.float64, device=dev)
+    tmax = torch.tensor([ms_rank], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+    pairs, poses, launches = (float(x) for x in tot.tolist())
+    ms = float(tmax.item())
+    value = pairs / (ms * 1e-3)
+    # dominant kernel (scoring): algorithmic pairs per launch / mean CUDA-event launch time
+    score_pairs_per_ms = st["pairs"] / st["score_ms"] if st["score_ms"] > 0 else 0.0
+    achieved = score_pairs_per_ms * 1e3 / 1e9           # Gpairs/s on this rank
+    pk = peaks()
+    f_max = pk.get("sm_max_mhz", 1965.0)
+    ops = OPS_CUTOFF if cutoff > 0 else OPS_ALLPAIRS
+    peak = N_SM * LANES * f_max * 1e6 / ops / 1e9
+    roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpairs/s", "frac": achieved / peak,
+            "traffic": ncu_traffic(args.config),
+            "peak_basis": f"{N_SM} SMs x {LANES} FP32 lanes x {f_max:.0f} MHz (MEASURED_PEAKS sm_max) / "
+                          f"{ops} canonical issue slots per pair",
+            "score_launches": st["score_launches"], "score_ms_total": st["score_ms"],
+            "score_share_of_step": st["score_ms"] / ms_rank if ms_rank > 0 else None}
+    if clk:
+        roof["frac_at_run_clock"] = achieved / (N_SM * LANES * clk["sm_mhz"] * 1e6 / ops / 1e9)
+
+    # ---- end to end through the public C ABI with host buffers (vs_create + vs_run + results to host)
+    e2e = None
+    if not args.no_e2e:
+        import torch as _t
+        pin = lambda a: _t.from_numpy(np.ascontiguousarray(a)).pin_memory().numpy()
+        host = [pin(x) for x in (prob.rec.xyz, prob.rec.q, prob.rec.type, prob.lig.xyz, prob.lig.q, prob.lig.type,
+                                 prob.spots)]
+        n_e2e = args.e2e_steps if args.e2e_steps is not None else max(1, min(args.steps, 2))
+        e2e_ctx_stats = []
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for i in range(n_e2e):
+            with vs.Context(*host, sp=sp, device=local) as c2:
+                c2.run(mp, args.seed + rank, None)
+                e2e_ctx_stats.append(c2.stats())
+        dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+        e2e_pairs = torch.tensor([sum(s["pairs"] for s in e2e_ctx_stats)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+            dist.all_reduce(e2e_pairs, op=dist.ReduceOp.SUM)
+        h2d = sum(a.nbytes for a in host)
+        d2h = n_spots * 8 * 4
+        e2e = {"value": float(e2e_pairs.item()) / float(dt.item()), "unit": "pairs/s", "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "steps": n_e2e,
+               "what": "vs_create (receptor/ligand/spot upload + per-spot list build) + vs_run (host spot ids) + "
+                       "best poses/scores to host, wall clock"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        lens = ctx.list_lengths()
+        n_s = 2
+        Gs = 2 if args.config in ("medium", "large", "sweep") else min(G, 5)
+        dt, pr, po, cores = oracle_sample(prob, {"cutoff": cutoff},
+                                          {"preset": args.preset, "population": cfg.population}, lens,
+                                          args.seed, n_s, Gs)
+        cpu = {"value": pr / dt, "unit": "pairs/s", "cores": cores, "kind": "oracle",
+               "sample": f"fp64 oracle vso_run, {n_s} spots x {Gs} generations of {args.config} "
+                         f"(P={cfg.population}, M{args.preset}), {po} poses, {dt:.1f} s; pairs counted as the "
+                         f"workload defines them (n_lig x list length), the oracle itself visits all n_rec atoms"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "pairs/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+            "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": args.config, "preset": f"M{args.preset}", "n_rec": cfg.n_rec, "n_lig": cfg.n_lig,
+                       "n_spots_per_rank": n_spots, "population": cfg.population, "generations": G,
+                       "mode": f"cutoff {cutoff:g} A, per-spot lists" if cutoff > 0 else "all pairs",
+                       "l2": "flushed between steps (256 MB write inside the timed region)",
+                       "parallelism": (f"dp{world}: independent runs per rank (seed+rank), best-of gathered"
+                                       if args.scaling == "weak" else
+                                       f"dp{world}: spots dealt by a dynamic chunk queue, one gather")},
+            "poses_per_s": poses / (ms * 1e-3),
+            "pairs_per_step": pairs / args.steps,
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": int(launches),
+            "clocks": clk,
+        }
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -35,6 +35,12 @@ extern "C" {
 
 #define VS_ABI_VERSION 1
 
+#if defined(__GNUC__)
+#define VS_API __attribute__((visibility("default")))
+#else
+#define VS_API
+#endif
+
 typedef struct vs_ctx vs_ctx; /* opaque; owned by the library */
 
 typedef enum {
@@ -85,7 +91,7 @@ typedef struct {
   float improve_frac, p_mut, mut_trans, mut_rot, ls_trans, ls_rot;
 } vs_mh_params;
 
-void vs_score_params_default(vs_score_params* out);
+VS_API void vs_score_params_default(vs_score_params* out);
 
 /* m = 1..4 -> M1..M4 of Table 4:
  *   M1 GA: P 64, f 0;  M2: P 64, f 1, L 8;  M3: P 64, f 0.2, L 8;
@@ -93,7 +99,7 @@ void vs_score_params_default(vs_score_params* out);
  *   G = 50 for M1-M3 (the paper does not report it, R22); p_mut 0.1,
  *   mut 1.0 A / 0.25, ls 0.5 A / 0.10.
  * Returns VS_ERR_INVALID_ARGUMENT for another m or out == NULL. */
-vs_status vs_mh_preset(int m, vs_mh_params* out);
+VS_API vs_status vs_mh_preset(int m, vs_mh_params* out);
 
 /* Builds a scoring context on CUDA device `cuda_device`.
  *   rec_xyz [n_rec][3], rec_q [n_rec], rec_type [n_rec]  receptor atoms
@@ -106,7 +112,7 @@ vs_status vs_mh_preset(int m, vs_mh_params* out);
  * spot centre, R10) are built on the device here.
  * Errors: VS_ERR_INVALID_ARGUMENT (NULL / counts / type ids / non-finite /
  * bad params), VS_ERR_CUDA, VS_ERR_OUT_OF_MEMORY.  *out = NULL on error. */
-vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec_type, int32_t n_rec,
+VS_API vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec_type, int32_t n_rec,
                     const float* lig_xyz, const float* lig_q, const int32_t* lig_type, int32_t n_lig,
                     const float* spot_xyz, int32_t n_spots, const vs_score_params* sp, int32_t cuda_device,
                     vs_ctx** out);
@@ -120,13 +126,13 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
  * n == 0 is a no-op.  Errors: VS_ERR_INVALID_ARGUMENT (NULL, n < 0, bad
  * spot id, non-finite), VS_ERR_ZERO_QUATERNION, VS_ERR_POSE_OUT_OF_REGION
  * (cutoff mode only), VS_ERR_CUDA. */
-vs_status vs_score_poses(vs_ctx* c, int64_t n, const int32_t* spot, const float* quat_wxyz, const float* trans,
+VS_API vs_status vs_score_poses(vs_ctx* c, int64_t n, const int32_t* spot, const float* quat_wxyz, const float* trans,
                          float* score_out);
 
 /* Same on device buffers, asynchronous on `cuda_stream` (a cudaStream_t;
  * NULL = legacy default stream).  Poses that fail validation get a NaN
  * score instead of an error status (no host round trip). */
-vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_quat,
+VS_API vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_quat,
                                 const float* d_trans, float* d_score, void* cuda_stream);
 
 /* Runs the metaheuristic independently at n_sel spots (synchronous).
@@ -136,18 +142,18 @@ vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_spot, con
  *   best_pose_out [n_sel][7] = (w,x,y,z,tx,ty,tz) of the best individual
  *   best_score_out [n_sel]   its score (fp32, kcal/mol)
  * Errors: VS_ERR_INVALID_ARGUMENT (params, ids), VS_ERR_CUDA, VS_ERR_OUT_OF_MEMORY. */
-vs_status vs_run(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+VS_API vs_status vs_run(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
                  float* best_pose_out, float* best_score_out);
 
 /* Same, asynchronous on `cuda_stream`; outputs in device memory.  spot_ids
  * is a HOST array (validated on the host).  The ctx's workspace is reused:
  * do not overlap two vs_run_async calls of one ctx on different streams. */
-vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+VS_API vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
                        float* d_best_pose, float* d_best_score, void* cuda_stream);
 
-void vs_destroy(vs_ctx* c); /* NULL-safe; synchronises the ctx's device work */
-const char* vs_last_error(void);
-int vs_abi_version(void);
+VS_API void vs_destroy(vs_ctx* c); /* NULL-safe; synchronises the ctx's device work */
+VS_API const char* vs_last_error(void);
+VS_API int vs_abi_version(void);
 
 /* ---- instrumentation ---------------------------------------------------- */
 typedef struct {
@@ -160,12 +166,12 @@ typedef struct {
 } vs_stats;
 
 /* enable = 1: bracket every scoring launch with CUDA events on its stream. */
-vs_status vs_set_timing(vs_ctx* c, int enable);
+VS_API vs_status vs_set_timing(vs_ctx* c, int enable);
 /* Synchronises the ctx's device and returns counters since the last reset. */
-vs_status vs_get_stats(vs_ctx* c, vs_stats* out);
-vs_status vs_reset_stats(vs_ctx* c);
+VS_API vs_status vs_get_stats(vs_ctx* c, vs_stats* out);
+VS_API vs_status vs_reset_stats(vs_ctx* c);
 /* Per-spot receptor list lengths (cutoff mode) or n_rec (all pairs). */
-vs_status vs_list_lengths(vs_ctx* c, int32_t* out /*[n_spots]*/);
+VS_API vs_status vs_list_lengths(vs_ctx* c, int32_t* out /*[n_spots]*/);
 
 /* ---- debug / lockstep trace -------------------------------------------- */
 typedef enum {
@@ -184,12 +190,12 @@ typedef void (*vs_trace_fn)(void* user, int32_t stage, int32_t g, int32_t l, int
                             const float* poses8, const int32_t* idx);
 
 /* vs_run with a callback after every stage (synchronises at each stage). */
-vs_status vs_run_trace(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+VS_API vs_status vs_run_trace(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
                        float* best_pose_out, float* best_score_out, vs_trace_fn fn, void* user);
 
 /* Device Philox4x32-10 for n counters: ctr [n][4], key [2] -> out [n][4]
  * (host buffers; for known-answer tests of the device generator). */
-vs_status vs_debug_philox(int64_t n, const uint32_t* ctr, const uint32_t* key, uint32_t* out);
+VS_API vs_status vs_debug_philox(int64_t n, const uint32_t* ctr, const uint32_t* key, uint32_t* out);
 
 #ifdef __cplusplus
 }

@@ -1,0 +1,764 @@
+// vs_api.cu -- C ABI (include/vs.h): context, validation, list building and the
+// device-resident generation loop of Algorithm 1.
+//
+// The paper's host loop copies the candidate set to each GPU and back for
+// every scoring call (Algorithm 2).  Here the whole population
+// lives in HBM for the run; the host only sequences kernel launches on one
+// stream, and the device boundary is crossed at the start (spot ids) and the
+// end (best pose + score per spot).
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/vs.h"
+#include "vs_kernels.cuh"
+
+using namespace vsk;
+
+namespace {
+
+thread_local std::string g_err;
+
+vs_status set_err(vs_status s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+
+// built-in atom types (R4/R5): C N O S H HD X
+const float kSigma[7] = {3.400f, 3.250f, 2.960f, 3.564f, 2.650f, 1.069f, 0.0f};
+const float kEps[7] = {0.1094f, 0.170f, 0.210f, 0.250f, 0.0157f, 0.0157f, 0.0f};
+const int kRole[7] = {0, 2, 2, 0, 0, 1, 0};
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t bytes) {
+    if (bytes <= cap) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e == cudaSuccess) cap = bytes;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
+           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_COUNT };
+
+bool finite_arr(const float* p, int64_t n) {
+  for (int64_t i = 0; i < n; ++i)
+    if (!std::isfinite(p[i])) return false;
+  return true;
+}
+
+}  // namespace
+
+struct vs_ctx {
+  int dev = 0;
+  int n_rec = 0, n_lig = 0, n_spots = 0;
+  bool all_pairs = false;
+  int dielectric = 0;
+  float T = 3.0f, rc = 0.0f, rc2 = INFINITY, inv_rc2 = 0.0f, r2min = 0.01f, hbC = 0.0f, hbD = 0.0f;
+  int n_groups = 0, n_chunks = 1;
+  std::vector<int> h_list_len;
+  int64_t list_total = 0;
+  RecAtom* d_lists = nullptr;
+  int* d_list_off = nullptr;
+  int* d_list_len = nullptr;
+  float4* d_shift = nullptr;
+  LigSlot* d_lig = nullptr;
+  int* d_iota = nullptr;
+  unsigned long long* d_counters = nullptr;
+  cudaStream_t stream = nullptr;
+  DevBuf buf[B_COUNT];
+  bool poisoned = false;
+  // instrumentation
+  uint64_t launches = 0, score_launches = 0;
+  bool timing = false;
+  std::vector<cudaEvent_t> ev;  // pairs (start, end)
+  size_t ev_used = 0;
+  double score_ms_acc = 0.0;
+  uint64_t timed_acc = 0;
+};
+
+namespace {
+
+vs_status cuda_fail(vs_ctx* c, cudaError_t e, const char* where) {
+  if (c) c->poisoned = true;
+  return set_err(e == cudaErrorMemoryAllocation ? VS_ERR_OUT_OF_MEMORY : VS_ERR_CUDA,
+                 std::string(where) + ": " + cudaGetErrorString(e));
+}
+
+#define CK(expr, where)                                 \
+  do {                                                  \
+    cudaError_t e_ = (expr);                            \
+    if (e_ != cudaSuccess) return cuda_fail(c, e_, where); \
+  } while (0)
+
+vs_status check_mh(const vs_mh_params* mp) {
+  if (!mp) return set_err(VS_ERR_INVALID_ARGUMENT, "mh params: NULL");
+  if (mp->population < 1 || mp->population > 2048) return set_err(VS_ERR_INVALID_ARGUMENT, "population must be in [1, 2048]");
+  if (mp->generations < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "generations must be >= 0");
+  if (mp->generations > 0 && mp->population < 2)
+    return set_err(VS_ERR_INVALID_ARGUMENT, "population must be >= 2 when generations > 0");
+  if (mp->ls_steps < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "ls_steps must be >= 0");
+  if (!(mp->improve_frac >= 0.0f && mp->improve_frac <= 1.0f)) return set_err(VS_ERR_INVALID_ARGUMENT, "improve_frac must be in [0, 1]");
+  if (!(mp->p_mut >= 0.0f && mp->p_mut <= 1.0f)) return set_err(VS_ERR_INVALID_ARGUMENT, "p_mut must be in [0, 1]");
+  const float st[4] = {mp->mut_trans, mp->mut_rot, mp->ls_trans, mp->ls_rot};
+  for (float v : st)
+    if (!(std::isfinite(v) && v >= 0.0f)) return set_err(VS_ERR_INVALID_ARGUMENT, "step sizes must be finite and >= 0");
+  return VS_OK;
+}
+
+// m = clamp(round-half-up(f * P), 1, P) with f the fp32 ABI value (R17)
+int improve_count(const vs_mh_params* mp) {
+  long long m = std::llround((double)mp->improve_frac * (double)mp->population);
+  if (m < 1) m = 1;
+  if (m > mp->population) m = mp->population;
+  return (int)m;
+}
+
+ScoreArgs base_args(vs_ctx* c) {
+  ScoreArgs a;
+  std::memset(&a, 0, sizeof(a));
+  a.lists = c->d_lists;
+  a.list_off = c->d_list_off;
+  a.list_len = c->d_list_len;
+  a.shift = c->d_shift;
+  a.lig = c->d_lig;
+  a.n_groups = c->n_groups;
+  a.n_chunks = c->n_chunks;
+  a.n_lig = c->n_lig;
+  a.r2min = c->r2min;
+  a.rc2 = c->rc2;
+  a.inv_rc2 = c->inv_rc2;
+  a.hbC = c->hbC;
+  a.hbD = c->hbD;
+  a.T = c->T;
+  a.counters = c->d_counters;
+  return a;
+}
+
+vs_status score_launch(vs_ctx* c, const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st) {
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (c->timing) {
+    if (c->ev_used + 2 > c->ev.size()) {
+      for (int i = 0; i < 64; ++i) {
+        cudaEvent_t e;
+        CK(cudaEventCreate(&e), "cudaEventCreate");
+        c->ev.push_back(e);
+      }
+    }
+    e0 = c->ev[c->ev_used];
+    e1 = c->ev[c->ev_used + 1];
+    c->ev_used += 2;
+    CK(cudaEventRecord(e0, st), "cudaEventRecord");
+  }
+  CK(launch_score(a, mode, !c->all_pairs, c->dielectric, n_blocks, st), "score kernel launch");
+  c->launches++;
+  c->score_launches++;
+  if (a.n_chunks > 1) {
+    CK(launch_finalize(a, mode, n_blocks, st), "finalize kernel launch");
+    c->launches++;
+  }
+  if (c->timing) CK(cudaEventRecord(e1, st), "cudaEventRecord");
+  return VS_OK;
+}
+
+vs_status collect_timing(vs_ctx* c) {
+  for (size_t i = 0; i + 1 < c->ev_used; i += 2) {
+    float ms = 0.0f;
+    CK(cudaEventSynchronize(c->ev[i + 1]), "cudaEventSynchronize");
+    CK(cudaEventElapsedTime(&ms, c->ev[i], c->ev[i + 1]), "cudaEventElapsedTime");
+    c->score_ms_acc += ms;
+    c->timed_acc++;
+  }
+  c->ev_used = 0;
+  return VS_OK;
+}
+
+struct Tracer {
+  vs_trace_fn fn = nullptr;
+  void* user = nullptr;
+  std::vector<float> hp;
+  std::vector<int32_t> hi;
+};
+
+vs_status trace_poses(vs_ctx* c, Tracer* tr, cudaStream_t st, int stage, int g, int l, int n_sel, int count,
+                      const PoseRec* d) {
+  if (!tr || !tr->fn) return VS_OK;
+  tr->hp.resize((size_t)n_sel * count * 8);
+  CK(cudaMemcpyAsync(tr->hp.data(), d, tr->hp.size() * sizeof(float), cudaMemcpyDeviceToHost, st), "trace D2H");
+  CK(cudaStreamSynchronize(st), "trace sync");
+  tr->fn(tr->user, stage, g, l, n_sel, count, tr->hp.data(), nullptr);
+  return VS_OK;
+}
+
+vs_status trace_idx(vs_ctx* c, Tracer* tr, cudaStream_t st, int stage, int g, int n_sel, int count, const int* d) {
+  if (!tr || !tr->fn) return VS_OK;
+  tr->hi.resize((size_t)n_sel * count);
+  CK(cudaMemcpyAsync(tr->hi.data(), d, tr->hi.size() * sizeof(int32_t), cudaMemcpyDeviceToHost, st), "trace D2H");
+  CK(cudaStreamSynchronize(st), "trace sync");
+  tr->fn(tr->user, stage, g, 0, n_sel, count, nullptr, tr->hi.data());
+  return VS_OK;
+}
+
+// The generation loop (Algorithm 1) for n_sel spots, all on stream st.
+vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                   float* d_best_pose, float* d_best_score, cudaStream_t st, Tracer* tr) {
+  vs_status s = check_mh(mp);
+  if (s != VS_OK) return s;
+  if (n_sel < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel must be >= 0");
+  if (!spot_ids && n_sel != 0 && n_sel != c->n_spots)
+    return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel must be 0 or n_spots when spot_ids is NULL");
+  if (spot_ids && n_sel == 0) return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel must be >= 1 with spot_ids");
+  const int ns = spot_ids ? n_sel : c->n_spots;
+  if (spot_ids)
+    for (int k = 0; k < ns; ++k)
+      if (spot_ids[k] < 0 || spot_ids[k] >= c->n_spots) return set_err(VS_ERR_INVALID_ARGUMENT, "spot id out of range");
+  const int P = mp->population;
+  const int m = improve_count(mp);
+  const bool improve = mp->improve_frac > 0.0f;
+  const size_t pop_bytes = sizeof(PoseRec) * (size_t)ns * P;
+  CK(c->buf[B_SEG].ensure(sizeof(int) * ns), "alloc");
+  CK(c->buf[B_SA].ensure(pop_bytes), "alloc");
+  CK(c->buf[B_SB].ensure(pop_bytes), "alloc");
+  CK(c->buf[B_C].ensure(pop_bytes), "alloc");
+  CK(c->buf[B_J].ensure(sizeof(int) * (size_t)ns * m), "alloc");
+  if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * (size_t)ns * P * c->n_chunks), "alloc");
+  int* seg = (int*)c->buf[B_SEG].p;
+  if (spot_ids)
+    CK(cudaMemcpyAsync(seg, spot_ids, sizeof(int) * ns, cudaMemcpyHostToDevice, st), "H2D spot ids");
+  else
+    CK(cudaMemcpyAsync(seg, c->d_iota, sizeof(int) * ns, cudaMemcpyDeviceToDevice, st), "D2D spot ids");
+  PoseRec* S = (PoseRec*)c->buf[B_SA].p;
+  PoseRec* S2 = (PoseRec*)c->buf[B_SB].p;
+  PoseRec* C = (PoseRec*)c->buf[B_C].p;
+  int* J = (int*)c->buf[B_J].p;
+
+  ScoreArgs plain = base_args(c);
+  plain.nseg = ns;
+  plain.seg_spot = seg;
+  plain.uniform = 1;
+  plain.seg_size = P;
+  plain.bps = (P + POSES_PER_CTA - 1) / POSES_PER_CTA;
+  plain.seg_stride = P;
+  plain.P = P;
+  plain.partial = (double*)c->buf[B_PART].p;
+  ScoreArgs ls = plain;
+  ls.seg_size = m;
+  ls.bps = (m + POSES_PER_CTA - 1) / POSES_PER_CTA;
+  ls.J = J;
+  ls.m = m;
+  ls.seed = seed;
+  ls.ls_trans = mp->ls_trans;
+  ls.ls_rot = mp->ls_rot;
+  const int plain_blocks = ns * plain.bps, ls_blocks = ns * ls.bps;
+
+  auto improve_step = [&](PoseRec* X, int g) -> vs_status {
+    CK(launch_popsort(0, X, nullptr, nullptr, J, ns, P, m, st), "select launch");
+    c->launches++;
+    vs_status r = trace_idx(c, tr, st, VS_TRACE_SELECT, g, ns, m, J);
+    if (r != VS_OK) return r;
+    for (int l = 0; l < mp->ls_steps; ++l) {
+      ScoreArgs a = ls;
+      a.poses = X;
+      a.g = g;
+      a.l = l;
+      r = score_launch(c, a, MODE_LS, ls_blocks, st);
+      if (r != VS_OK) return r;
+      r = trace_poses(c, tr, st, VS_TRACE_LS, g, l, ns, P, X);
+      if (r != VS_OK) return r;
+    }
+    return VS_OK;
+  };
+
+  // Initialize(S)
+  CK(launch_init(S, ns, P, seg, seed, c->T, st), "init launch");
+  c->launches++;
+  vs_status r = trace_poses(c, tr, st, VS_TRACE_INIT, 0, 0, ns, P, S);
+  if (r != VS_OK) return r;
+  {
+    ScoreArgs a = plain;
+    a.poses = S;
+    if ((r = score_launch(c, a, MODE_PLAIN, plain_blocks, st)) != VS_OK) return r;
+  }
+  if ((r = trace_poses(c, tr, st, VS_TRACE_SCORED, 0, 0, ns, P, S)) != VS_OK) return r;
+  if (improve && (r = improve_step(S, 0)) != VS_OK) return r;
+  CK(launch_popsort(1, S, nullptr, S2, nullptr, ns, P, m, st), "sort launch");
+  c->launches++;
+  std::swap(S, S2);
+  if ((r = trace_poses(c, tr, st, VS_TRACE_SORTED, 0, 0, ns, P, S)) != VS_OK) return r;
+  // while !End(S): Select, Combine, Improve, Include
+  for (int g = 1; g <= mp->generations; ++g) {
+    CK(launch_combine(S, C, ns, P, seg, seed, g, mp->p_mut, mp->mut_trans, mp->mut_rot, c->T, st), "combine launch");
+    c->launches++;
+    if ((r = trace_poses(c, tr, st, VS_TRACE_COMBINED, g, 0, ns, P, C)) != VS_OK) return r;
+    ScoreArgs a = plain;
+    a.poses = C;
+    if ((r = score_launch(c, a, MODE_PLAIN, plain_blocks, st)) != VS_OK) return r;
+    if ((r = trace_poses(c, tr, st, VS_TRACE_SCORED, g, 0, ns, P, C)) != VS_OK) return r;
+    if (improve && (r = improve_step(C, g)) != VS_OK) return r;
+    CK(launch_popsort(2, S, C, S2, nullptr, ns, P, m, st), "include launch");
+    c->launches++;
+    std::swap(S, S2);
+    if ((r = trace_poses(c, tr, st, VS_TRACE_INCLUDED, g, 0, ns, P, S)) != VS_OK) return r;
+  }
+  CK(launch_best(S, ns, P, d_best_pose, d_best_score, st), "best launch");
+  c->launches++;
+  return VS_OK;
+}
+
+vs_status score_device_impl(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_q, const float* d_t,
+                            float* d_out, cudaStream_t st) {
+  if (n == 0) return VS_OK;
+  const int ns = c->n_spots;
+  CK(c->buf[B_VALID].ensure(sizeof(int) * n), "alloc");
+  CK(c->buf[B_COUNTS].ensure(sizeof(int) * ns), "alloc");
+  CK(c->buf[B_PP].ensure(sizeof(int) * (ns + 1)), "alloc");
+  CK(c->buf[B_BP].ensure(sizeof(int) * (ns + 1)), "alloc");
+  CK(c->buf[B_CUR].ensure(sizeof(int) * ns), "alloc");
+  CK(c->buf[B_SORTED].ensure(sizeof(PoseRec) * n), "alloc");
+  CK(c->buf[B_ORIG].ensure(sizeof(int) * n), "alloc");
+  if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * n * c->n_chunks), "alloc");
+  int* valid = (int*)c->buf[B_VALID].p;
+  int* counts = (int*)c->buf[B_COUNTS].p;
+  int* pp = (int*)c->buf[B_PP].p;
+  int* bp = (int*)c->buf[B_BP].p;
+  int* cur = (int*)c->buf[B_CUR].p;
+  PoseRec* sorted = (PoseRec*)c->buf[B_SORTED].p;
+  int* orig = (int*)c->buf[B_ORIG].p;
+  CK(cudaMemsetAsync(counts, 0, sizeof(int) * ns, st), "memset");
+  CK(launch_validate(n, d_spot, d_q, d_t, ns, c->T, c->all_pairs ? 0 : 1, valid, counts, d_out, st), "validate launch");
+  CK(launch_scan(counts, ns, pp, bp, cur, st), "scan launch");
+  CK(launch_scatter(n, d_spot, d_q, d_t, valid, cur, sorted, orig, st), "scatter launch");
+  c->launches += 3;
+  ScoreArgs a = base_args(c);
+  a.nseg = ns;
+  a.seg_spot = c->d_iota;
+  a.uniform = 0;
+  a.blk_prefix = bp;
+  a.pose_prefix = pp;
+  a.poses = sorted;
+  a.orig = orig;
+  a.score_out = d_out;
+  a.partial = (double*)c->buf[B_PART].p;
+  const int64_t blocks = (n + POSES_PER_CTA - 1) / POSES_PER_CTA + ns;
+  if (blocks > 0x7fffffff) return set_err(VS_ERR_INVALID_ARGUMENT, "too many poses in one call");
+  return score_launch(c, a, MODE_PLAIN, (int)blocks, st);
+}
+
+}  // namespace
+
+extern "C" {
+
+void vs_score_params_default(vs_score_params* o) {
+  if (!o) return;
+  o->coulomb_k = 332.0636f;
+  o->dielectric = 0;
+  o->eps_r = 1.0f;
+  o->cutoff = 12.0f;
+  o->region_half_width = 3.0f;
+  o->hb_eps = 5.0f;
+  o->hb_r0 = 1.9f;
+  o->r2_min = 0.01f;
+  o->n_types = 0;
+  o->type_sigma = nullptr;
+  o->type_eps = nullptr;
+  o->type_hb_role = nullptr;
+}
+
+vs_status vs_mh_preset(int m, vs_mh_params* o) {
+  if (!o) return set_err(VS_ERR_INVALID_ARGUMENT, "out: NULL");
+  if (m < 1 || m > 4) return set_err(VS_ERR_INVALID_ARGUMENT, "preset must be 1..4 (Table 4: M1..M4)");
+  o->population = m == 4 ? 1024 : 64;
+  o->generations = m == 4 ? 0 : 50;
+  o->ls_steps = m == 1 ? 0 : 8;
+  o->improve_frac = m == 1 ? 0.0f : (m == 3 ? 0.2f : 1.0f);
+  o->p_mut = 0.1f;
+  o->mut_trans = 1.0f;
+  o->mut_rot = 0.25f;
+  o->ls_trans = 0.5f;
+  o->ls_rot = 0.10f;
+  return VS_OK;
+}
+
+vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec_type, int32_t n_rec,
+                    const float* lig_xyz, const float* lig_q, const int32_t* lig_type, int32_t n_lig,
+                    const float* spot_xyz, int32_t n_spots, const vs_score_params* sp_in, int32_t cuda_device,
+                    vs_ctx** out) {
+  if (!out) return set_err(VS_ERR_INVALID_ARGUMENT, "out: NULL");
+  *out = nullptr;
+  if (!rec_xyz || !rec_q || !rec_type || !lig_xyz || !lig_q || !lig_type || !spot_xyz)
+    return set_err(VS_ERR_INVALID_ARGUMENT, "NULL input array");
+  if (n_rec < 1 || n_lig < 1 || n_lig > 256 || n_spots < 1)
+    return set_err(VS_ERR_INVALID_ARGUMENT, "need n_rec >= 1, 1 <= n_lig <= 256, n_spots >= 1");
+  vs_score_params sp;
+  if (sp_in) sp = *sp_in; else vs_score_params_default(&sp);
+  if (!std::isfinite(sp.coulomb_k) || (sp.dielectric != 0 && sp.dielectric != 1) ||
+      (sp.dielectric == 1 && !(sp.eps_r > 0.0f && std::isfinite(sp.eps_r))) ||
+      !(sp.region_half_width > 0.0f && std::isfinite(sp.region_half_width)) ||
+      !(sp.hb_eps >= 0.0f && std::isfinite(sp.hb_eps)) || !(sp.hb_r0 > 0.0f && std::isfinite(sp.hb_r0)) ||
+      !(sp.r2_min > 0.0f && std::isfinite(sp.r2_min)) || std::isnan(sp.cutoff))
+    return set_err(VS_ERR_INVALID_ARGUMENT, "invalid score params");
+  if (sp.n_types < 0 || sp.n_types > 64 || (sp.n_types > 0 && (!sp.type_sigma || !sp.type_eps || !sp.type_hb_role)))
+    return set_err(VS_ERR_INVALID_ARGUMENT, "invalid type table");
+  if (!finite_arr(rec_xyz, 3 * (int64_t)n_rec) || !finite_arr(rec_q, n_rec) || !finite_arr(lig_xyz, 3 * (int64_t)n_lig) ||
+      !finite_arr(lig_q, n_lig) || !finite_arr(spot_xyz, 3 * (int64_t)n_spots))
+    return set_err(VS_ERR_INVALID_ARGUMENT, "non-finite input");
+  const int nt = sp.n_types > 0 ? sp.n_types : 7;
+  std::vector<float> c12(nt), c6(nt), don(nt), acc(nt);
+  for (int t = 0; t < nt; ++t) {
+    const float sg = sp.n_types > 0 ? sp.type_sigma[t] : kSigma[t];
+    const float ep = sp.n_types > 0 ? sp.type_eps[t] : kEps[t];
+    const int rl = sp.n_types > 0 ? sp.type_hb_role[t] : kRole[t];
+    if (!(sg >= 0.0f && std::isfinite(sg)) || !(ep >= 0.0f && std::isfinite(ep)) || rl < 0 || rl > 2)
+      return set_err(VS_ERR_INVALID_ARGUMENT, "invalid type table entry");
+    // geometric combining: 4 eps_ij (sig_ij^12/r^12 - sig_ij^6/r^6) = c12_i c12_j/r^12 - c6_i c6_j/r^6 (R4)
+    c12[t] = (float)(2.0 * std::sqrt((double)ep) * std::pow((double)sg, 6));
+    c6[t] = (float)(2.0 * std::sqrt((double)ep) * std::pow((double)sg, 3));
+    don[t] = rl == 1 ? 1.0f : 0.0f;
+    acc[t] = rl == 2 ? 1.0f : 0.0f;
+  }
+  for (int i = 0; i < n_rec; ++i)
+    if (rec_type[i] < 0 || rec_type[i] >= nt) return set_err(VS_ERR_INVALID_ARGUMENT, "receptor type id out of range");
+  for (int i = 0; i < n_lig; ++i)
+    if (lig_type[i] < 0 || lig_type[i] >= nt) return set_err(VS_ERR_INVALID_ARGUMENT, "ligand type id out of range");
+
+  int ndev = 0;
+  cudaError_t e0 = cudaGetDeviceCount(&ndev);
+  if (e0 != cudaSuccess || ndev == 0)
+    return set_err(VS_ERR_CUDA, std::string("no CUDA device: ") + cudaGetErrorString(e0));
+  if (cuda_device < 0 || cuda_device >= ndev) return set_err(VS_ERR_INVALID_ARGUMENT, "cuda_device out of range");
+
+  vs_ctx* c = new (std::nothrow) vs_ctx;
+  if (!c) return set_err(VS_ERR_OUT_OF_MEMORY, "out of host memory");
+  DeviceGuard guard(cuda_device);
+  c->dev = cuda_device;
+  c->n_rec = n_rec;
+  c->n_lig = n_lig;
+  c->n_spots = n_spots;
+  c->all_pairs = !(sp.cutoff > 0.0f) || std::isinf(sp.cutoff);
+  c->dielectric = sp.dielectric;
+  c->T = sp.region_half_width;
+  c->rc = c->all_pairs ? INFINITY : sp.cutoff;
+  c->rc2 = c->all_pairs ? INFINITY : (float)((double)sp.cutoff * sp.cutoff);
+  c->inv_rc2 = c->all_pairs ? 0.0f : (float)(1.0 / ((double)sp.cutoff * sp.cutoff));
+  c->r2min = sp.r2_min;
+  c->hbC = (float)(5.0 * sp.hb_eps * std::pow((double)sp.hb_r0, 12));
+  c->hbD = (float)(6.0 * sp.hb_eps * std::pow((double)sp.hb_r0, 10));
+
+  auto fail = [&](vs_status s) {
+    vs_destroy(c);
+    return s;
+  };
+#define CKC(expr, where)                                     \
+  do {                                                       \
+    cudaError_t e_ = (expr);                                 \
+    if (e_ != cudaSuccess) return fail(cuda_fail(nullptr, e_, where)); \
+  } while (0)
+
+  CKC(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking), "stream create");
+  // ligand: centred on the fp32-rounded fp64 centroid (R11); slots in K_SLOTS groups
+  float cen[3];
+  for (int a = 0; a < 3; ++a) {
+    double s = 0.0;
+    for (int i = 0; i < n_lig; ++i) s += lig_xyz[3 * i + a];
+    cen[a] = (float)(s / n_lig);
+  }
+  c->n_groups = (n_lig + K_SLOTS - 1) / K_SLOTS;
+  c->n_chunks = (c->n_groups + GROUPS_PER_CTA - 1) / GROUPS_PER_CTA;
+  const int n_slot_groups = c->n_chunks > 1 ? c->n_chunks * GROUPS_PER_CTA : c->n_groups;
+  std::vector<LigSlot> slots((size_t)n_slot_groups * K_SLOTS);
+  std::memset(slots.data(), 0, sizeof(LigSlot) * slots.size());
+  double rmax = 0.0;
+  for (int i = 0; i < n_lig; ++i) {
+    const int t = lig_type[i];
+    LigSlot& s = slots[i];
+    s.lq.x = lig_xyz[3 * i] - cen[0];
+    s.lq.y = lig_xyz[3 * i + 1] - cen[1];
+    s.lq.z = lig_xyz[3 * i + 2] - cen[2];
+    const double qk = sp.dielectric == 0 ? (double)sp.coulomb_k * lig_q[i] / 4.0
+                                         : (double)sp.coulomb_k * lig_q[i] / (double)sp.eps_r;
+    s.lq.w = (float)qk;
+    s.p = make_float4(c12[t], c6[t], don[t], acc[t]);
+    rmax = std::max(rmax, std::sqrt((double)s.lq.x * s.lq.x + (double)s.lq.y * s.lq.y + (double)s.lq.z * s.lq.z));
+  }
+  CKC(cudaMalloc(&c->d_lig, sizeof(LigSlot) * slots.size()), "alloc ligand");
+  CKC(cudaMemcpy(c->d_lig, slots.data(), sizeof(LigSlot) * slots.size(), cudaMemcpyHostToDevice), "H2D ligand");
+
+  // receptor atoms (absolute) + per-atom parameters
+  std::vector<float4> hrec(n_rec), hprm(n_rec);
+  double c0d[3] = {0, 0, 0};
+  for (int j = 0; j < n_rec; ++j) {
+    const int t = rec_type[j];
+    hrec[j] = make_float4(rec_xyz[3 * j], rec_xyz[3 * j + 1], rec_xyz[3 * j + 2], rec_q[j]);
+    hprm[j] = make_float4(c12[t], c6[t], don[t], acc[t]);
+    for (int a = 0; a < 3; ++a) c0d[a] += rec_xyz[3 * j + a];
+  }
+  float4* d_rec = nullptr;
+  float4* d_prm = nullptr;
+  float4* d_centres = nullptr;
+  auto free_tmp = [&]() {
+    if (d_rec) cudaFree(d_rec);
+    if (d_prm) cudaFree(d_prm);
+    if (d_centres) cudaFree(d_centres);
+  };
+#define CKT(expr, where)                                                       \
+  do {                                                                         \
+    cudaError_t e_ = (expr);                                                   \
+    if (e_ != cudaSuccess) { free_tmp(); return fail(cuda_fail(nullptr, e_, where)); } \
+  } while (0)
+  CKT(cudaMalloc(&d_rec, sizeof(float4) * n_rec), "alloc receptor");
+  CKT(cudaMalloc(&d_prm, sizeof(float4) * n_rec), "alloc receptor");
+  CKT(cudaMemcpy(d_rec, hrec.data(), sizeof(float4) * n_rec, cudaMemcpyHostToDevice), "H2D receptor");
+  CKT(cudaMemcpy(d_prm, hprm.data(), sizeof(float4) * n_rec, cudaMemcpyHostToDevice), "H2D receptor");
+
+  std::vector<int> h_off(n_spots), h_len(n_spots), iota(n_spots);
+  std::vector<float4> h_shift(n_spots);
+  for (int s = 0; s < n_spots; ++s) iota[s] = s;
+  if (c->all_pairs) {
+    // one list: whole receptor relative to its fp32 centroid c0; pose origin shifted by c_s - c0
+    float c0[3] = {(float)(c0d[0] / n_rec), (float)(c0d[1] / n_rec), (float)(c0d[2] / n_rec)};
+    float4 hc = make_float4(c0[0], c0[1], c0[2], 0.0f);
+    CKT(cudaMalloc(&d_centres, sizeof(float4)), "alloc");
+    CKT(cudaMemcpy(d_centres, &hc, sizeof(float4), cudaMemcpyHostToDevice), "H2D");
+    CKT(cudaMalloc(&c->d_lists, sizeof(RecAtom) * n_rec), "alloc lists");
+    int zero = 0;
+    CKT(cudaMalloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
+    CKT(cudaMemcpy(c->d_list_off, &zero, sizeof(int), cudaMemcpyHostToDevice), "H2D");
+    CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, 1, INFINITY, c->d_list_off, nullptr, c->d_lists, 0,
+                           c->stream), "list fill launch");
+    for (int s = 0; s < n_spots; ++s) {
+      h_off[s] = 0;
+      h_len[s] = n_rec;
+      h_shift[s] = make_float4(spot_xyz[3 * s] - c0[0], spot_xyz[3 * s + 1] - c0[1], spot_xyz[3 * s + 2] - c0[2], 0.0f);
+    }
+    c->list_total = n_rec;
+  } else {
+    // per-spot lists: atoms within T sqrt(3) + max|l_i| + rc + 0.01 of the spot centre (R10)
+    const double reach = (double)c->T * std::sqrt(3.0) + rmax + (double)sp.cutoff + 0.01;
+    std::vector<float4> hc(n_spots);
+    for (int s = 0; s < n_spots; ++s) hc[s] = make_float4(spot_xyz[3 * s], spot_xyz[3 * s + 1], spot_xyz[3 * s + 2], 0.0f);
+    CKT(cudaMalloc(&d_centres, sizeof(float4) * n_spots), "alloc");
+    CKT(cudaMemcpy(d_centres, hc.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
+    CKT(cudaMalloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
+    CKT(cudaMalloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
+    CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, (float)(reach * reach), nullptr, c->d_list_len,
+                           nullptr, 1, c->stream), "list count launch");
+    CKT(cudaMemcpyAsync(h_len.data(), c->d_list_len, sizeof(int) * n_spots, cudaMemcpyDeviceToHost, c->stream), "D2H");
+    CKT(cudaStreamSynchronize(c->stream), "sync");
+    int64_t tot = 0;
+    for (int s = 0; s < n_spots; ++s) {
+      h_off[s] = (int)tot;
+      tot += h_len[s];
+      h_shift[s] = make_float4(0, 0, 0, 0);
+    }
+    if (tot > 0x7fffffff) { free_tmp(); return fail(set_err(VS_ERR_OUT_OF_MEMORY, "receptor lists exceed 2^31 atoms")); }
+    c->list_total = tot;
+    CKT(cudaMalloc(&c->d_lists, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
+    CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+    CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, (float)(reach * reach), c->d_list_off, nullptr,
+                           c->d_lists, 0, c->stream), "list fill launch");
+  }
+  if (!c->d_list_len) CKT(cudaMalloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
+  CKT(cudaMemcpy(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+  CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+  CKT(cudaMalloc(&c->d_shift, sizeof(float4) * n_spots), "alloc");
+  CKT(cudaMemcpy(c->d_shift, h_shift.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
+  CKT(cudaMalloc(&c->d_iota, sizeof(int) * n_spots), "alloc");
+  CKT(cudaMemcpy(c->d_iota, iota.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+  CKT(cudaMalloc(&c->d_counters, sizeof(unsigned long long) * 2), "alloc");
+  CKT(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 2), "memset");
+  CKT(cudaStreamSynchronize(c->stream), "sync");
+  free_tmp();
+  c->h_list_len = h_len;
+  c->launches = 0;
+  *out = c;
+  return VS_OK;
+#undef CKT
+#undef CKC
+}
+
+vs_status vs_score_poses(vs_ctx* c, int64_t n, const int32_t* spot, const float* q, const float* t, float* out) {
+  if (!c) return set_err(VS_ERR_INVALID_ARGUMENT, "ctx: NULL");
+  if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
+  if (n < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "n must be >= 0");
+  if (n == 0) return VS_OK;
+  if (!spot || !q || !t || !out) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL pose array");
+  for (int64_t p = 0; p < n; ++p) {
+    if (spot[p] < 0 || spot[p] >= c->n_spots) return set_err(VS_ERR_INVALID_ARGUMENT, "spot id out of range");
+    if (!finite_arr(q + 4 * p, 4) || !finite_arr(t + 3 * p, 3)) return set_err(VS_ERR_INVALID_ARGUMENT, "non-finite pose");
+    if (q[4 * p] == 0.0f && q[4 * p + 1] == 0.0f && q[4 * p + 2] == 0.0f && q[4 * p + 3] == 0.0f)
+      return set_err(VS_ERR_ZERO_QUATERNION, "zero quaternion");
+    if (!c->all_pairs)
+      for (int a = 0; a < 3; ++a)
+        if (std::fabs(t[3 * p + a]) > c->T) return set_err(VS_ERR_POSE_OUT_OF_REGION, "translation outside the spot region");
+  }
+  DeviceGuard guard(c->dev);
+  cudaStream_t st = c->stream;
+  CK(c->buf[B_SPOT].ensure(sizeof(int32_t) * n), "alloc");
+  CK(c->buf[B_Q].ensure(sizeof(float) * 4 * n), "alloc");
+  CK(c->buf[B_T].ensure(sizeof(float) * 3 * n), "alloc");
+  CK(c->buf[B_OUT].ensure(sizeof(float) * n), "alloc");
+  CK(cudaMemcpyAsync(c->buf[B_SPOT].p, spot, sizeof(int32_t) * n, cudaMemcpyHostToDevice, st), "H2D");
+  CK(cudaMemcpyAsync(c->buf[B_Q].p, q, sizeof(float) * 4 * n, cudaMemcpyHostToDevice, st), "H2D");
+  CK(cudaMemcpyAsync(c->buf[B_T].p, t, sizeof(float) * 3 * n, cudaMemcpyHostToDevice, st), "H2D");
+  vs_status s = score_device_impl(c, n, (const int32_t*)c->buf[B_SPOT].p, (const float*)c->buf[B_Q].p,
+                                  (const float*)c->buf[B_T].p, (float*)c->buf[B_OUT].p, st);
+  if (s != VS_OK) return s;
+  CK(cudaMemcpyAsync(out, c->buf[B_OUT].p, sizeof(float) * n, cudaMemcpyDeviceToHost, st), "D2H");
+  CK(cudaStreamSynchronize(st), "sync");
+  return VS_OK;
+}
+
+vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_q, const float* d_t,
+                                float* d_score, void* stream) {
+  if (!c) return set_err(VS_ERR_INVALID_ARGUMENT, "ctx: NULL");
+  if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
+  if (n < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "n must be >= 0");
+  if (n == 0) return VS_OK;
+  if (!d_spot || !d_q || !d_t || !d_score) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL pose array");
+  DeviceGuard guard(c->dev);
+  return score_device_impl(c, n, d_spot, d_q, d_t, d_score, (cudaStream_t)stream);
+}
+
+static vs_status run_host(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                          float* best_pose, float* best_score, Tracer* tr) {
+  if (!c) return set_err(VS_ERR_INVALID_ARGUMENT, "ctx: NULL");
+  if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
+  if (!best_pose || !best_score) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL output");
+  DeviceGuard guard(c->dev);
+  const int ns = spot_ids ? n_sel : c->n_spots;
+  if (ns < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel must be >= 0");
+  CK(c->buf[B_BEST].ensure(sizeof(float) * 7 * std::max(ns, 1)), "alloc");
+  CK(c->buf[B_BESTS].ensure(sizeof(float) * std::max(ns, 1)), "alloc");
+  vs_status s = run_impl(c, mp, seed, n_sel, spot_ids, (float*)c->buf[B_BEST].p, (float*)c->buf[B_BESTS].p,
+                         c->stream, tr);
+  if (s != VS_OK) return s;
+  CK(cudaMemcpyAsync(best_pose, c->buf[B_BEST].p, sizeof(float) * 7 * ns, cudaMemcpyDeviceToHost, c->stream), "D2H");
+  CK(cudaMemcpyAsync(best_score, c->buf[B_BESTS].p, sizeof(float) * ns, cudaMemcpyDeviceToHost, c->stream), "D2H");
+  CK(cudaStreamSynchronize(c->stream), "sync");
+  return VS_OK;
+}
+
+vs_status vs_run(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                 float* best_pose_out, float* best_score_out) {
+  return run_host(c, mp, seed, n_sel, spot_ids, best_pose_out, best_score_out, nullptr);
+}
+
+vs_status vs_run_trace(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                       float* best_pose_out, float* best_score_out, vs_trace_fn fn, void* user) {
+  Tracer tr;
+  tr.fn = fn;
+  tr.user = user;
+  return run_host(c, mp, seed, n_sel, spot_ids, best_pose_out, best_score_out, &tr);
+}
+
+vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
+                       float* d_best_pose, float* d_best_score, void* stream) {
+  if (!c) return set_err(VS_ERR_INVALID_ARGUMENT, "ctx: NULL");
+  if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
+  if (!d_best_pose || !d_best_score) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL output");
+  DeviceGuard guard(c->dev);
+  return run_impl(c, mp, seed, n_sel, spot_ids, d_best_pose, d_best_score, (cudaStream_t)stream, nullptr);
+}
+
+void vs_destroy(vs_ctx* c) {
+  if (!c) return;
+  DeviceGuard guard(c->dev);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  cudaDeviceSynchronize();
+  for (auto& b : c->buf) b.release();
+  for (auto e : c->ev) cudaEventDestroy(e);
+  void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_lig, c->d_iota, c->d_counters};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+  if (c->stream) cudaStreamDestroy(c->stream);
+  delete c;
+}
+
+const char* vs_last_error(void) { return g_err.c_str(); }
+int vs_abi_version(void) { return VS_ABI_VERSION; }
+
+vs_status vs_set_timing(vs_ctx* c, int enable) {
+  if (!c) return set_err(VS_ERR_INVALID_ARGUMENT, "ctx: NULL");
+  c->timing = enable != 0;
+  return VS_OK;
+}
+
+vs_status vs_get_stats(vs_ctx* c, vs_stats* o) {
+  if (!c || !o) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
+  DeviceGuard guard(c->dev);
+  CK(cudaDeviceSynchronize(), "sync");
+  vs_status s = collect_timing(c);
+  if (s != VS_OK) return s;
+  unsigned long long h[2];
+  CK(cudaMemcpy(h, c->d_counters, sizeof(h), cudaMemcpyDeviceToHost), "D2H counters");
+  o->kernel_launches = c->launches;
+  o->score_launches = c->score_launches;
+  o->pairs = h[0];
+  o->poses_scored = h[1];
+  o->score_ms = c->score_ms_acc;
+  o->timed_launches = c->timed_acc;
+  return VS_OK;
+}
+
+vs_status vs_reset_stats(vs_ctx* c) {
+  if (!c) return set_err(VS_ERR_INVALID_ARGUMENT, "ctx: NULL");
+  if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
+  DeviceGuard guard(c->dev);
+  CK(cudaDeviceSynchronize(), "sync");
+  CK(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 2), "memset");
+  c->ev_used = 0;
+  c->launches = c->score_launches = 0;
+  c->score_ms_acc = 0.0;
+  c->timed_acc = 0;
+  return VS_OK;
+}
+
+vs_status vs_list_lengths(vs_ctx* c, int32_t* out) {
+  if (!c || !out) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL argument");
+  std::memcpy(out, c->h_list_len.data(), sizeof(int32_t) * c->n_spots);
+  return VS_OK;
+}
+
+vs_status vs_debug_philox(int64_t n, const uint32_t* ctr, const uint32_t* key, uint32_t* out) {
+  if (n < 0 || (n > 0 && (!ctr || !key || !out))) return set_err(VS_ERR_INVALID_ARGUMENT, "bad arguments");
+  if (n == 0) return VS_OK;
+  vs_ctx* c = nullptr;
+  uint4 *dc = nullptr, *dout = nullptr;
+  CK(cudaMalloc(&dc, sizeof(uint4) * n), "alloc");
+  cudaError_t e = cudaMalloc(&dout, sizeof(uint4) * n);
+  if (e == cudaSuccess) e = cudaMemcpy(dc, ctr, sizeof(uint4) * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = launch_philox(n, dc, make_uint2(key[0], key[1]), dout, nullptr);
+  if (e == cudaSuccess) e = cudaMemcpy(out, dout, sizeof(uint4) * n, cudaMemcpyDeviceToHost);
+  cudaFree(dc);
+  if (dout) cudaFree(dout);
+  if (e != cudaSuccess) return cuda_fail(c, e, "debug philox");
+  return VS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,76 @@
+// vs_kernels.cuh -- launch-side declarations shared by vs_score.cu, vs_pop.cu, vs_api.cu.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "vs_device.cuh"
+
+namespace vsk {
+
+constexpr int K_SLOTS = 8;          // ligand atoms per thread (register blocking)
+constexpr int GROUPS_PER_CTA = 8;   // warps (ligand-atom groups) per CTA at most
+constexpr int POSES_PER_CTA = 32;   // one pose per lane
+constexpr int TILE = 128;           // receptor atoms per shared-memory stage (4 KB)
+constexpr int NSTAGE = 4;           // bulk-copy ring depth
+
+enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
+
+// Work decomposition of one scoring launch: segments (one spot each) of poses,
+// split into 32-pose blocks; blockIdx.y = ligand group chunk.
+struct ScoreArgs {
+  // receptor lists (per spot) and ligand slots
+  const RecAtom* lists;
+  const int* list_off;
+  const int* list_len;
+  const float4* shift;       // added to t + R l (all-pairs: c_s - c0; cutoff: 0)
+  const LigSlot* lig;
+  int n_groups;              // ligand groups of K_SLOTS slots
+  int n_chunks;              // ceil(n_groups / GROUPS_PER_CTA)
+  int n_lig;                 // real ligand atoms (pair accounting)
+  float r2min, rc2, inv_rc2; // rc2 = +inf in all-pairs mode
+  float hbC, hbD;
+  // segments
+  int nseg;
+  const int* seg_spot;       // [nseg] global spot id
+  int uniform;               // 1: every segment has seg_size poses
+  int seg_size, bps;         // uniform
+  const int* blk_prefix;     // non-uniform: [nseg+1]
+  const int* pose_prefix;    // non-uniform: [nseg+1]
+  // PLAIN
+  PoseRec* poses;            // segment k pose p at k*seg_stride + p (uniform) or pose_prefix[k] + p
+  int seg_stride;
+  const int* orig;           // optional: original index of each pose -> score_out
+  float* score_out;
+  double* partial;           // n_chunks > 1: [n_poses_total][n_chunks]
+  // LS (Improve step): X[k*P + J[k*m + jj]] perturbed, scored, accepted if better
+  const int* J;
+  int m, P;
+  uint64_t seed;
+  int g, l;
+  float ls_trans, ls_rot, T;
+  unsigned long long* counters;  // [0] pairs, [1] poses
+};
+
+// launchers (return cudaError_t of the launch)
+cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectric, int n_blocks, cudaStream_t st);
+cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st);
+cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, uint64_t seed, float T, cudaStream_t st);
+cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, uint64_t seed, int g,
+                           float p_mut, float mut_trans, float mut_rot, float T, cudaStream_t st);
+// sort (score, index) per segment: mode 0: select best m indices -> J;
+// mode 1: sort S -> S_out; mode 2: include: best P of S ++ C -> S_out
+cudaError_t launch_popsort(int mode, const PoseRec* S, const PoseRec* C, PoseRec* S_out, int* J, int n_sel, int P,
+                           int m, cudaStream_t st);
+cudaError_t launch_best(const PoseRec* S, int n_sel, int P, float* best_pose, float* best_score, cudaStream_t st);
+cudaError_t launch_build_lists(const float4* rec, const float4* rprm, int n_rec, const float4* spot_c, int n_spots,
+                               float reach2, const int* off, int* len, RecAtom* lists, int count_only,
+                               cudaStream_t st);
+cudaError_t launch_philox(int64_t n, const uint4* ctr, uint2 key, uint4* out, cudaStream_t st);
+// vs_score_poses helpers
+cudaError_t launch_validate(int64_t n, const int32_t* spot, const float* q, const float* t, int n_spots, float T,
+                            int cutoff, int* valid, int* counts, float* score_out, cudaStream_t st);
+cudaError_t launch_scan(const int* counts, int n, int* pose_prefix, int* blk_prefix, int* cursor, cudaStream_t st);
+cudaError_t launch_scatter(int64_t n, const int32_t* spot, const float* q, const float* t, const int* valid,
+                           int* cursor, PoseRec* sorted, int* orig, cudaStream_t st);
+
+}  // namespace vsk

@@ -1,0 +1,344 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Bars (BASELINE.json north_star):
+  * scores: |gpu - oracle| <= max(1e-4 |oracle|, 1e-3 kcal/mol) per pose;
+  * pose generation from a Philox stream: bit-exact;
+  * vs_run best score within 1e-3 relative of the oracle on identical streams.
+Decisions taken on scores (Improve's accept, sorts) are checked exactly against
+the GPU's own fp32 scores, and against the oracle's fp64 scores except at near
+ties (|gap| below the per-pose tolerance), where both outcomes are correct.
+"""
+import math
+
+import numpy as np
+import pytest
+
+from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
+
+pytestmark = pytest.mark.gpu
+
+
+def tol(ref):
+    return np.maximum(1e-4 * np.abs(ref), 1e-3)
+
+
+def assert_scores(gpu, ref, what=""):
+    gpu = np.asarray(gpu, np.float64)
+    ref = np.asarray(ref, np.float64)
+    err = np.abs(gpu - ref)
+    bad = err > tol(ref)
+    assert not bad.any(), f"{what}: {bad.sum()} / {len(ref)} poses out of tolerance; worst err/tol " \
+                          f"{(err / tol(ref)).max():.3g} at {int(np.argmax(err / tol(ref)))}"
+    return float((err / tol(ref)).max())
+
+
+@pytest.fixture(scope="module")
+def gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    vs.load()
+    return torch
+
+
+def both(oracle_mod, prob, cutoff=12.0, ligand=None, **kw):
+    sp_o = oracle_mod.score_params(cutoff=cutoff, **kw)
+    sp_g = vs.score_params(cutoff=cutoff, **kw)
+    return (vs.Context.from_problem(prob, sp_g, ligand=ligand),
+            oracle_mod.Oracle.from_problem(prob, sp_o, ligand=ligand))
+
+
+# ------------------------------------------------------------------ RNG
+def test_device_philox_known_answers(gpu, oracle_mod):
+    kat = [([0, 0, 0, 0], [0, 0], [0x6627e8d5, 0xe169c58d, 0xbc57ac4c, 0x9b00dbd8]),
+           ([0xffffffff] * 4, [0xffffffff] * 2, [0x408f276d, 0x41c83b0e, 0xa20bc7c6, 0x6d5451fd]),
+           ([0x243f6a88, 0x85a308d3, 0x13198a2e, 0x03707344], [0xa4093822, 0x299f31d0],
+            [0xd16cfe09, 0x94fdcceb, 0x5001e420, 0x24126ea1])]
+    for ctr, key, want in kat:
+        assert list(vs.debug_philox([ctr], key)[0]) == want
+    rng = np.random.default_rng(0)
+    ctr = rng.integers(0, 2 ** 32, size=(4096, 4), dtype=np.uint64).astype(np.uint32)
+    key = [0x12345678, 0x9abcdef0]
+    got = vs.debug_philox(ctr, key)
+    for i in range(0, 4096, 97):
+        assert list(got[i]) == list(oracle_mod.philox(ctr[i], key))
+
+
+# ------------------------------------------------------------------ scoring parity
+@pytest.mark.parametrize("cutoff", [12.0, 0.0])
+@pytest.mark.parametrize("name", ["tiny", "small"])
+def test_score_parity_all_poses(gpu, oracle_mod, name, cutoff):
+    prob = synth.make_problem(name)
+    g, o = both(oracle_mod, prob, cutoff)
+    n = 300 if name == "tiny" else 96
+    spot, q, t = synth.make_poses(n, prob.cfg.n_spots, 3.0, seed=17)
+    # mix in near-contact poses: scaled-down translations towards the spot atom
+    t[: n // 3] *= 0.2
+    assert_scores(g.score_poses(spot, q, t), o.score(spot, q, t), f"{name} rc={cutoff}")
+
+
+@pytest.mark.parametrize("name", ["medium", "large"])
+def test_score_parity_sampled_full_size(gpu, oracle_mod, name):
+    """Full-size problem, large batch through the GPU; the oracle checks a sample."""
+    prob = synth.make_problem(name)
+    g, o = both(oracle_mod, prob, 12.0)
+    n = 20000
+    spot, q, t = synth.make_poses(n, prob.cfg.n_spots, 3.0, seed=5)
+    got = g.score_poses(spot, q, t)
+    idx = np.random.default_rng(1).choice(n, 12, replace=False)
+    assert_scores(got[idx], o.score(spot[idx], q[idx], t[idx]), name)
+    assert np.all(np.isfinite(got))
+
+
+@pytest.mark.parametrize("n_lig", [1, 7, 9, 64, 65, 100, 256])
+def test_ragged_ligand_sizes(gpu, oracle_mod, n_lig):
+    """Ligands that are not a multiple of the 8-atom register block, and > 64 atoms (chunked CTAs)."""
+    prob = synth.make_custom(1500, n_lig, 5, seed=n_lig)
+    for cutoff in (12.0, 0.0):
+        g, o = both(oracle_mod, prob, cutoff)
+        spot, q, t = synth.make_poses(70, 5, 3.0, seed=3)
+        assert_scores(g.score_poses(spot, q, t), o.score(spot, q, t), f"n_lig={n_lig} rc={cutoff}")
+
+
+def test_list_tiles_ragged_and_empty(gpu, oracle_mod):
+    """Spot far outside the receptor (empty cutoff list) and list lengths across tile boundaries."""
+    prob = synth.make_custom(700, 13, 4, seed=2)
+    prob.spots[3] = prob.spots[3] + np.float32(80.0)   # nothing within reach
+    g, o = both(oracle_mod, prob, 12.0)
+    lens = g.list_lengths()
+    assert lens[3] == 0 and lens[:3].min() > 128
+    spot, q, t = synth.make_poses(64, 4, 3.0, seed=8)
+    got = g.score_poses(spot, q, t)
+    assert np.all(got[spot == 3] == 0.0)
+    assert_scores(got, o.score(spot, q, t))
+
+
+def test_binned_lists_equal_all_pairs_cutoff(gpu, oracle_mod):
+    """Binning is exact: per-spot lists give the brute-force cutoff score for in-region poses,
+    including poses on the region boundary."""
+    prob = synth.make_problem("small")
+    g, o = both(oracle_mod, prob, 12.0)
+    spot, q, t = synth.make_poses(64, prob.cfg.n_spots, 3.0, seed=4)
+    t[:16] = np.sign(t[:16]) * np.float32(3.0)   # corners of the region box
+    assert_scores(g.score_poses(spot, q, t), o.score(spot, q, t))
+
+
+def test_quaternion_conventions_on_gpu(gpu, oracle_mod):
+    prob = synth.make_problem("tiny")
+    g, o = both(oracle_mod, prob, 0.0)
+    spot, q, t = synth.make_poses(40, 4, 3.0, seed=6)
+    a = g.score_poses(spot, q, t)
+    b = g.score_poses(spot, -q, t)
+    c = g.score_poses(spot, 4.0 * q, t)
+    assert_scores(a, o.score(spot, q, t))
+    assert_scores(b, o.score(spot, q, t))
+    assert_scores(c, o.score(spot, q, t))
+
+
+@pytest.mark.parametrize("kw", [dict(dielectric=1, eps_r=4.0), dict(hb_eps=0.0), dict(r2_min=0.25)])
+def test_score_param_variants(gpu, oracle_mod, kw):
+    prob = synth.make_problem("tiny")
+    for cutoff in (12.0, 0.0):
+        g, o = both(oracle_mod, prob, cutoff, **kw)
+        spot, q, t = synth.make_poses(128, 4, 3.0, seed=12)
+        assert_scores(g.score_poses(spot, q, t), o.score(spot, q, t), str(kw))
+
+
+def test_custom_type_table(gpu, oracle_mod):
+    import ctypes as C
+    prob = synth.make_problem("tiny")
+    sig = np.array([3.1, 2.8, 2.2, 3.0, 2.0, 1.2, 0.5], np.float32)
+    eps = np.array([0.2, 0.1, 0.3, 0.05, 0.02, 0.01, 0.0], np.float32)
+    role = np.array([0, 1, 2, 2, 0, 1, 0], np.int32)
+    kw = dict(n_types=7, type_sigma=sig.ctypes.data_as(C.POINTER(C.c_float)),
+              type_eps=eps.ctypes.data_as(C.POINTER(C.c_float)), type_hb_role=role.ctypes.data_as(C.POINTER(C.c_int)))
+    g, o = both(oracle_mod, prob, 12.0, **kw)
+    spot, q, t = synth.make_poses(100, 4, 3.0, seed=2)
+    assert_scores(g.score_poses(spot, q, t), o.score(spot, q, t))
+
+
+def test_score_errors_and_empty(gpu, oracle_mod):
+    prob = synth.make_problem("tiny")
+    g, _ = both(oracle_mod, prob, 12.0)
+    assert len(g.score_poses(np.zeros(0, np.int32), np.zeros((0, 4)), np.zeros((0, 3)))) == 0
+    cases = [([0], [[0, 0, 0, 0]], [[0, 0, 0]], vs.ERR_ZERO_QUATERNION),
+             ([0], [[1, 0, 0, 0]], [[0, 3.01, 0]], vs.ERR_POSE_OUT_OF_REGION),
+             ([4], [[1, 0, 0, 0]], [[0, 0, 0]], vs.ERR_INVALID_ARGUMENT),
+             ([0], [[1, 0, np.nan, 0]], [[0, 0, 0]], vs.ERR_INVALID_ARGUMENT)]
+    for s, q, t, code in cases:
+        with pytest.raises(vs.VSError) as e:
+            g.score_poses(np.array(s, np.int32), np.array(q, np.float32), np.array(t, np.float32))
+        assert e.value.status == code
+    # the ctx stays usable after argument errors
+    assert np.isfinite(g.score_poses(np.array([1], np.int32), np.array([[1, 0, 0, 0]], np.float32),
+                                     np.zeros((1, 3), np.float32)))[0]
+
+
+def test_device_entry_point(gpu, oracle_mod):
+    torch = gpu
+    prob = synth.make_problem("small")
+    g, o = both(oracle_mod, prob, 12.0)
+    spot, q, t = synth.make_poses(5000, prob.cfg.n_spots, 3.0, seed=21)
+    q[7] = 0.0            # invalid -> NaN
+    t[8, 0] = 9.0         # out of region -> NaN
+    spot[9] = 999         # bad spot -> NaN
+    spot_d = torch.from_numpy(np.where(spot < prob.cfg.n_spots, spot, 0)).cuda()
+    spot_d[9] = 999
+    qd, td = torch.from_numpy(q).cuda(), torch.from_numpy(t).cuda()
+    out = torch.zeros(5000, device="cuda")
+    g.score_poses_device(spot_d, qd, td, out)
+    torch.cuda.synchronize()
+    res = out.cpu().numpy()
+    assert np.isnan(res[[7, 8, 9]]).all()
+    ok = np.setdiff1d(np.arange(5000), [7, 8, 9])
+    host = g.score_poses(spot[ok], q[ok], t[ok])
+    np.testing.assert_array_equal(res[ok], host)            # same kernel, same bits
+    idx = ok[::250]
+    assert_scores(res[idx], o.score(spot[idx], q[idx], t[idx]))
+
+
+def test_stats_count_pairs(gpu, oracle_mod):
+    prob = synth.make_problem("tiny")
+    g, _ = both(oracle_mod, prob, 12.0)
+    g.reset_stats()
+    g.set_timing(True)
+    spot, q, t = synth.make_poses(100, 4, 3.0, seed=2)
+    g.score_poses(spot, q, t)
+    st = g.stats()
+    lens = g.list_lengths()
+    assert st["poses_scored"] == 100
+    assert st["pairs"] == int(sum(lens[s] for s in spot)) * prob.cfg.n_lig
+    assert st["score_launches"] == 1 and st["timed_launches"] == 1 and st["score_ms"] > 0
+
+
+# ------------------------------------------------------------------ metaheuristic
+def _run_pair(oracle_mod, name="tiny", cutoff=12.0):
+    prob = synth.make_problem(name)
+    return prob, both(oracle_mod, prob, cutoff)
+
+
+def test_run_free_running_matches_oracle(gpu, oracle_mod):
+    prob, (g, o) = _run_pair(oracle_mod)
+    for m in (1, 2, 3):
+        mp_g = vs.mh_preset(m, population=prob.cfg.population, generations=prob.cfg.generations)
+        mp_o = oracle_mod.mh_preset(m, population=prob.cfg.population, generations=prob.cfg.generations)
+        pg, sg = g.run(mp_g, 42)
+        po, so = o.run(mp_o, 42)
+        rel = np.abs(sg - so) / np.maximum(np.abs(so), 1e-3)
+        assert np.all(rel <= 1e-3), (m, sg, so)
+
+
+def test_run_m4_neighbourhood(gpu, oracle_mod):
+    prob, (g, o) = _run_pair(oracle_mod)
+    pg, sg = g.run(vs.mh_preset(4, population=128), 3)
+    po, so = o.run(oracle_mod.mh_preset(4, population=128), 3)
+    assert np.all(np.abs(sg - so) <= 1e-3 * np.maximum(np.abs(so), 1.0))
+
+
+def test_run_g0_f0_reduces_to_min_of_scored_initial_poses(gpu, oracle_mod):
+    prob, (g, o) = _run_pair(oracle_mod)
+    P = 32
+    pose, best = g.run(vs.mh_preset(1, population=P, generations=0), 9)
+    init = np.array([[o.init_pose(9, s, i) for i in range(P)] for s in range(4)])
+    for s in range(4):
+        sc = g.score_poses(np.full(P, s, np.int32), init[s, :, :4], init[s, :, 4:])
+        k = int(np.argmin(sc))
+        assert best[s] == sc[k]                      # identical kernel arithmetic -> identical bits
+        np.testing.assert_array_equal(pose[s], init[s, k])
+
+
+def test_run_deterministic_and_chunk_independent(gpu, oracle_mod):
+    prob, (g, _) = _run_pair(oracle_mod, "small")
+    mp = vs.mh_preset(3, population=64, generations=4)
+    p1, s1 = g.run(mp, 5)
+    p2, s2 = g.run(mp, 5)
+    np.testing.assert_array_equal(p1, p2)
+    np.testing.assert_array_equal(s1, s2)
+    ids = np.arange(prob.cfg.n_spots, dtype=np.int32)[::-1].copy()
+    parts = [g.run(mp, 5, ids[a:a + 23]) for a in range(0, len(ids), 23)]
+    pc = np.concatenate([p for p, _ in parts])
+    sc = np.concatenate([s for _, s in parts])
+    np.testing.assert_array_equal(pc, p1[ids])
+    np.testing.assert_array_equal(sc, s1[ids])
+
+
+def test_run_errors(gpu, oracle_mod):
+    prob, (g, _) = _run_pair(oracle_mod)
+    with pytest.raises(vs.VSError):
+        g.run(vs.mh_preset(1, population=1, generations=2), 1)
+    with pytest.raises(vs.VSError):
+        g.run(vs.mh_preset(1), 1, np.array([7], np.int32))
+    with pytest.raises(vs.VSError):
+        g.run(vs.mh_preset(1, population=4096), 1)
+
+
+@pytest.mark.parametrize("preset,P,G", [(3, 32, 4), (2, 16, 2), (4, 64, 0)])
+def test_lockstep_trace(gpu, oracle_mod, preset, P, G):
+    """Every stage of Algorithm 1 on the GPU re-derived by the oracle from the GPU's own state:
+    pose generation byte-exact, decisions exact on GPU scores, scores within tolerance."""
+    prob, (g, o) = _run_pair(oracle_mod)
+    seed = 77
+    mp_g = vs.mh_preset(preset, population=P, generations=G)
+    mp_o = oracle_mod.mh_preset(preset, population=P, generations=G)
+    m = oracle_mod.improve_count(mp_o)
+    events = []
+    g.run_trace(mp_g, seed, None, lambda *e: events.append(e))
+    spots = range(prob.cfg.n_spots)
+    prev = None       # population before the current stage
+    sorted_S = None
+    J = None
+    n_near_ties = 0
+    for stage, gen, l, pop, idx in events:
+        if stage == vs.TRACE_INIT:
+            for s in spots:
+                for i in range(P):
+                    np.testing.assert_array_equal(pop[s, i, :7], o.init_pose(seed, s, i))
+            prev = pop
+        elif stage == vs.TRACE_COMBINED:
+            for s in spots:
+                for j in range(P):
+                    want = o.combine_child(mp_o, seed, s, gen, j, sorted_S[s, :, :7])
+                    np.testing.assert_array_equal(pop[s, j, :7], want)
+            prev = pop
+        elif stage == vs.TRACE_SCORED:
+            for s in spots:
+                np.testing.assert_array_equal(pop[s, :, :7], prev[s, :, :7])
+                assert_scores(pop[s, :, 7], o.score(np.full(P, s, np.int32), pop[s, :, :4], pop[s, :, 4:7]))
+            prev = pop
+        elif stage == vs.TRACE_SELECT:
+            for s in spots:
+                np.testing.assert_array_equal(idx[s], oracle_mod.select_improve(prev[s, :, 7].astype(np.float64), m))
+            J = idx
+        elif stage == vs.TRACE_LS:
+            for s in spots:
+                js = set(J[s].tolist())
+                for j in range(P):
+                    if j not in js:
+                        np.testing.assert_array_equal(pop[s, j], prev[s, j])
+                        continue
+                    prop = o.ls_proposal(mp_o, seed, s, gen, l, j, prev[s, j, :7])
+                    accepted = not np.array_equal(pop[s, j], prev[s, j])
+                    e_prop = o.score_one(s, prop[:4], prop[4:])
+                    e_old = o.score_one(s, prev[s, j, :4], prev[s, j, 4:7])
+                    if accepted:
+                        np.testing.assert_array_equal(pop[s, j, :7], prop)
+                        assert pop[s, j, 7] < prev[s, j, 7]
+                        assert_scores([pop[s, j, 7]], [e_prop])
+                    if accepted != (e_prop < e_old):
+                        assert abs(e_prop - e_old) <= 2 * tol(e_old), (s, j, e_prop, e_old)
+                        n_near_ties += 1
+            prev = pop
+        elif stage == vs.TRACE_SORTED:
+            for s in spots:
+                order = np.argsort(prev[s, :, 7], kind="stable")
+                np.testing.assert_array_equal(pop[s], prev[s, order])
+            sorted_S = pop
+            prev = pop
+        elif stage == vs.TRACE_INCLUDED:
+            for s in spots:
+                origin = oracle_mod.include(sorted_S[s, :, 7].astype(np.float64), prev[s, :, 7].astype(np.float64))
+                both_pop = np.concatenate([sorted_S[s], prev[s]])
+                np.testing.assert_array_equal(pop[s], both_pop[origin])
+            sorted_S = pop
+            prev = pop
+    assert n_near_ties <= 2
