@@ -80,7 +80,7 @@ struct vs_ctx {
   bool all_pairs = false;
   int dielectric = 0;
   float T = 3.0f, rc = 0.0f, rc2 = INFINITY, inv_rc2 = 0.0f, r2min = 0.01f, hbC = 0.0f, hbD = 0.0f;
-  int n_groups = 0, n_chunks = 1;
+  int n_groups = 0, n_chunks = 1, hb_start = 0;
   std::vector<int> h_list_len;
   int64_t list_total = 0;
   RecAtom* d_lists = nullptr;
@@ -148,6 +148,7 @@ ScoreArgs base_args(vs_ctx* c) {
   a.shift = c->d_shift;
   a.lig = c->d_lig;
   a.n_groups = c->n_groups;
+  a.hb_start = c->hb_start;
   a.n_chunks = c->n_chunks;
   a.n_lig = c->n_lig;
   a.r2min = c->r2min;
@@ -487,15 +488,23 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     for (int i = 0; i < n_lig; ++i) s += lig_xyz[3 * i + a];
     cen[a] = (float)(s / n_lig);
   }
-  c->n_groups = (n_lig + K_SLOTS - 1) / K_SLOTS;
-  c->n_chunks = (c->n_groups + GROUPS_PER_CTA - 1) / GROUPS_PER_CTA;
-  const int n_slot_groups = c->n_chunks > 1 ? c->n_chunks * GROUPS_PER_CTA : c->n_groups;
-  std::vector<LigSlot> slots((size_t)n_slot_groups * K_SLOTS);
+  // slot order: atoms without an H-bond role first, then donors/acceptors, as
+  // float2 slot pairs; padding pairs (all-zero dummy atoms, exactly 0 energy) sit in between so
+  // that every H-bond pair is in the tail of the slot sequence (hb_start).
+  std::vector<int> plain, hbat;
+  for (int i = 0; i < n_lig; ++i) (don[lig_type[i]] != 0.0f || acc[lig_type[i]] != 0.0f ? hbat : plain).push_back(i);
+  const int pairs_plain = ((int)plain.size() + 1) / 2, pairs_hb = ((int)hbat.size() + 1) / 2;
+  const int groups = (pairs_plain + pairs_hb + K_PAIRS - 1) / K_PAIRS;
+  c->n_chunks = (groups + GROUPS_PER_CTA - 1) / GROUPS_PER_CTA;
+  c->n_groups = c->n_chunks > 1 ? c->n_chunks * GROUPS_PER_CTA : groups;
+  const int pairs_tot = c->n_groups * K_PAIRS;
+  c->hb_start = pairs_tot - pairs_hb;
+  std::vector<LigSlot> slots((size_t)pairs_tot * 2);
   std::memset(slots.data(), 0, sizeof(LigSlot) * slots.size());
   double rmax = 0.0;
-  for (int i = 0; i < n_lig; ++i) {
+  auto put = [&](int slot, int i) {
     const int t = lig_type[i];
-    LigSlot& s = slots[i];
+    LigSlot& s = slots[slot];
     s.lq.x = lig_xyz[3 * i] - cen[0];
     s.lq.y = lig_xyz[3 * i + 1] - cen[1];
     s.lq.z = lig_xyz[3 * i + 2] - cen[2];
@@ -504,18 +513,18 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     s.lq.w = (float)qk;
     s.p = make_float4(c12[t], c6[t], don[t], acc[t]);
     rmax = std::max(rmax, std::sqrt((double)s.lq.x * s.lq.x + (double)s.lq.y * s.lq.y + (double)s.lq.z * s.lq.z));
-  }
+  };
+  for (size_t a = 0; a < plain.size(); ++a) put((int)a, plain[a]);
+  for (size_t a = 0; a < hbat.size(); ++a) put(2 * c->hb_start + (int)a, hbat[a]);
   CKC(cudaMalloc(&c->d_lig, sizeof(LigSlot) * slots.size()), "alloc ligand");
   CKC(cudaMemcpy(c->d_lig, slots.data(), sizeof(LigSlot) * slots.size(), cudaMemcpyHostToDevice), "H2D ligand");
 
   // receptor atoms (absolute) + per-atom parameters
   std::vector<float4> hrec(n_rec), hprm(n_rec);
-  double c0d[3] = {0, 0, 0};
   for (int j = 0; j < n_rec; ++j) {
     const int t = rec_type[j];
     hrec[j] = make_float4(rec_xyz[3 * j], rec_xyz[3 * j + 1], rec_xyz[3 * j + 2], rec_q[j]);
     hprm[j] = make_float4(c12[t], c6[t], don[t], acc[t]);
-    for (int a = 0; a < 3; ++a) c0d[a] += rec_xyz[3 * j + a];
   }
   float4* d_rec = nullptr;
   float4* d_prm = nullptr;
@@ -539,23 +548,25 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   std::vector<float4> h_shift(n_spots);
   for (int s = 0; s < n_spots; ++s) iota[s] = s;
   if (c->all_pairs) {
-    // one list: whole receptor relative to its fp32 centroid c0; pose origin shifted by c_s - c0
-    float c0[3] = {(float)(c0d[0] / n_rec), (float)(c0d[1] / n_rec), (float)(c0d[2] / n_rec)};
-    float4 hc = make_float4(c0[0], c0[1], c0[2], 0.0f);
-    CKT(cudaMalloc(&d_centres, sizeof(float4)), "alloc");
-    CKT(cudaMemcpy(d_centres, &hc, sizeof(float4), cudaMemcpyHostToDevice), "H2D");
-    CKT(cudaMalloc(&c->d_lists, sizeof(RecAtom) * n_rec), "alloc lists");
-    int zero = 0;
-    CKT(cudaMalloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
-    CKT(cudaMemcpy(c->d_list_off, &zero, sizeof(int), cudaMemcpyHostToDevice), "H2D");
-    CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, 1, INFINITY, c->d_list_off, nullptr, c->d_lists, 0,
-                           c->stream), "list fill launch");
+    // every spot streams the whole receptor, stored relative to the spot centre (fp32 r_j - c_s,
+    // the same relative frame as the cutoff lists: keeps the pair differences accurate)
+    std::vector<float4> hc(n_spots);
+    for (int s = 0; s < n_spots; ++s) hc[s] = make_float4(spot_xyz[3 * s], spot_xyz[3 * s + 1], spot_xyz[3 * s + 2], 0.0f);
+    CKT(cudaMalloc(&d_centres, sizeof(float4) * n_spots), "alloc");
+    CKT(cudaMemcpy(d_centres, hc.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
+    const int64_t tot = (int64_t)n_rec * n_spots;
+    if (tot > 0x7fffffff) { free_tmp(); return fail(set_err(VS_ERR_OUT_OF_MEMORY, "receptor lists exceed 2^31 atoms")); }
     for (int s = 0; s < n_spots; ++s) {
-      h_off[s] = 0;
+      h_off[s] = (int)((int64_t)s * n_rec);
       h_len[s] = n_rec;
-      h_shift[s] = make_float4(spot_xyz[3 * s] - c0[0], spot_xyz[3 * s + 1] - c0[1], spot_xyz[3 * s + 2] - c0[2], 0.0f);
+      h_shift[s] = make_float4(0, 0, 0, 0);
     }
-    c->list_total = n_rec;
+    CKT(cudaMalloc(&c->d_lists, sizeof(RecAtom) * tot), "alloc lists");
+    CKT(cudaMalloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
+    CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+    CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, INFINITY, c->d_list_off, nullptr, c->d_lists, 0,
+                           c->stream), "list fill launch");
+    c->list_total = tot;
   } else {
     // per-spot lists: atoms within T sqrt(3) + max|l_i| + rc + 0.01 of the spot centre (R10)
     const double reach = (double)c->T * std::sqrt(3.0) + rmax + (double)sp.cutoff + 0.01;

@@ -8,6 +8,7 @@
 namespace vsk {
 
 constexpr int K_SLOTS = 8;          // ligand atoms per thread (register blocking)
+constexpr int K_PAIRS = K_SLOTS / 2; // slot pairs: one float2 lane-pair per FFMA2
 constexpr int GROUPS_PER_CTA = 8;   // warps (ligand-atom groups) per CTA at most
 constexpr int POSES_PER_CTA = 32;   // one pose per lane
 constexpr int TILE = 128;           // receptor atoms per shared-memory stage (4 KB)
@@ -25,6 +26,7 @@ struct ScoreArgs {
   const float4* shift;       // added to t + R l (all-pairs: c_s - c0; cutoff: 0)
   const LigSlot* lig;
   int n_groups;              // ligand groups of K_SLOTS slots
+  int hb_start;              // first slot pair with hydrogen-bond atoms (pairs before it: no HB)
   int n_chunks;              // ceil(n_groups / GROUPS_PER_CTA)
   int n_lig;                 // real ligand atoms (pair accounting)
   float r2min, rc2, inv_rc2; // rc2 = +inf in all-pairs mode

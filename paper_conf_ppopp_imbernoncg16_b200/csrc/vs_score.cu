@@ -4,17 +4,23 @@
 //
 // Layout of one CTA:
 //   lane  = one pose of a 32-pose block of one spot;
-//   warp  = one group of K_SLOTS ligand atoms (transformed coordinates and the
-//           per-atom accumulators Q, A, B, H6, H5 live in registers);
+//   warp  = one group of K_SLOTS ligand atoms, held as K_PAIRS float2 slot
+//           pairs: transformed coordinates and the per-atom accumulators live
+//           in registers and every fp32 add/mul/fma of the pair loop is a
+//           packed FADD2/FMUL2/FFMA2 over two ligand atoms, with the receptor
+//           atom's value as the broadcast operand;
 //   the spot's receptor list streams through a NSTAGE-deep shared-memory ring
 //   filled by the bulk-copy (TMA) engine; every lane reads the same receptor
 //   atom (warp-uniform broadcast LDS.128).
+// Ligand atoms are ordered on the host so that hydrogen-bond-capable atoms
+// (donor HD, acceptor N/O; R5) come last: a group's first K_PAIRS - H pairs
+// skip the H-bond arithmetic, and H (warp-uniform) selects a specialised loop.
 // Energy of slot i after the sweep over the list:
 //   E_i = es_i Q_i + c12_i A_i - c6_i B_i + C H6_i - D H5_i
-//   Q_i = sum_j q_j S(r2)/r2 (DDD) , A_i = sum_j c12_j / r^12, B_i = sum_j c6_j / r^6,
+//   Q_i = sum_j q_j S(r2)/r2 (DDD), A_i = sum_j c12_j / r^12, B_i = sum_j c6_j / r^6,
 //   H6_i = sum_j w_ij / r^12, H5_i = sum_j w_ij / r^10.
-// The per-pose sum over slots and warps is done in a fixed order
-// (deterministic: identical poses give identical fp32 scores).
+// The per-slot combination and the per-pose sum over slots and warps run in
+// fp64 in a fixed order (deterministic: identical poses -> identical scores).
 #include "vs_kernels.cuh"
 
 namespace vsk {
@@ -31,6 +37,91 @@ __device__ __forceinline__ void locate(const ScoreArgs& a, int bx, int& k, int& 
     }
     k = lo;
     blk = bx - __ldg(a.blk_prefix + k);
+  }
+}
+
+__device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
+
+struct Acc {
+  float2 X[K_PAIRS], Y[K_PAIRS], Z[K_PAIRS];
+  float2 Q[K_PAIRS], A[K_PAIRS], B[K_PAIRS];
+  float2 H6[K_PAIRS], H5[K_PAIRS];
+  float2 DN[K_PAIRS], AC[K_PAIRS];
+};
+
+// Sweep of the spot's receptor list for one warp whose group has H H-bond pairs.
+template <int H, bool CUT, int DIEL>
+__device__ __forceinline__ void sweep(Acc& r, RecAtom (*tile)[TILE], uint64_t* full, const RecAtom* src, int len,
+                                      int nt, float r2min, float rc2, float inv_rc2) {
+  const float INF = __int_as_float(0x7f800000);
+  for (int it = 0; it < nt; ++it) {
+    const int st = it % NSTAGE;
+    mbar_wait(&full[st], (uint32_t)(it / NSTAGE) & 1u);
+    const int nvalid = min(TILE, len - it * TILE);
+    const RecAtom* T = tile[st];
+#pragma unroll 2
+    for (int j = 0; j < nvalid; ++j) {
+      const float4 xq = T[j].xq;
+      const float4 pp = T[j].p;
+#pragma unroll
+      for (int p = 0; p < K_PAIRS; ++p) {
+        const float2 dx = __fadd2_rn(r.X[p], f2(-xq.x));
+        const float2 dy = __fadd2_rn(r.Y[p], f2(-xq.y));
+        const float2 dz = __fadd2_rn(r.Z[p], f2(-xq.z));
+        float2 r2 = __fmul2_rn(dx, dx);
+        r2 = __ffma2_rn(dy, dy, r2);
+        r2 = __ffma2_rn(dz, dz, r2);
+        r2.x = fmaxf(r2.x, r2min);                                   // R7
+        r2.y = fmaxf(r2.y, r2min);
+        bool inx = true, iny = true;
+        float2 r2u = r2;
+        if (CUT) {
+          inx = r2.x < rc2;
+          iny = r2.y < rc2;
+          r2.x = inx ? r2.x : INF;                                   // beyond rc: 1/r2 -> 0
+          r2.y = iny ? r2.y : INF;
+        }
+        float2 inv;
+        inv.x = rcp_approx(r2.x);
+        inv.y = rcp_approx(r2.y);
+        float2 es = inv;
+        if (DIEL == 0) {
+          // shifted DDD Coulomb (R6): S(r2)/r2 = (1 - r2/rc2)^2 / r2 = 1/r2 - 2/rc2 + r2/rc2^2
+          if (CUT) {
+            es = __fadd2_rn(__ffma2_rn(r2u, f2(inv_rc2 * inv_rc2), inv), f2(-2.0f * inv_rc2));
+            es.x = inx ? es.x : 0.0f;
+            es.y = iny ? es.y : 0.0f;
+          }
+        } else {
+          es.x = rsqrt_approx(r2.x);
+          es.y = rsqrt_approx(r2.y);
+          if (CUT) {
+            const float2 sh = __ffma2_rn(r2u, f2(-inv_rc2), f2(1.0f));   // 1 - r2/rc2
+            es = __fmul2_rn(__fmul2_rn(es, sh), sh);
+          }
+        }
+        r.Q[p] = __ffma2_rn(es, f2(xq.w), r.Q[p]);
+        const float2 inv2 = __fmul2_rn(inv, inv);
+        const float2 inv3 = __fmul2_rn(inv2, inv);
+        const float2 inv6 = __fmul2_rn(inv3, inv3);
+        r.A[p] = __ffma2_rn(inv6, f2(pp.x), r.A[p]);
+        r.B[p] = __ffma2_rn(inv3, f2(pp.y), r.B[p]);
+        if (p >= K_PAIRS - H) {                                      // compile-time after unrolling
+          const float2 inv5 = __fmul2_rn(inv3, inv2);
+          // donor slot pairs with receptor acceptors, acceptor slot with receptor donors (R5)
+          const float2 w = make_float2(r.DN[p].x != 0.0f ? pp.w : pp.z, r.DN[p].y != 0.0f ? pp.w : pp.z);
+          r.H6[p] = __ffma2_rn(w, inv6, r.H6[p]);
+          r.H5[p] = __ffma2_rn(w, inv5, r.H5[p]);
+        }
+      }
+    }
+    __syncthreads();  // every warp is done with stage st
+    if (threadIdx.x == 0 && it + NSTAGE < nt) {
+      const int nx = it + NSTAGE;
+      const uint32_t bytes = (uint32_t)min(TILE, len - nx * TILE) * (uint32_t)sizeof(RecAtom);
+      mbar_arrive_expect_tx(&full[st], bytes);
+      bulk_g2s(tile[st], src + (size_t)nx * TILE, bytes, &full[st]);
+    }
   }
 }
 
@@ -53,6 +144,7 @@ __global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const Sco
   const bool active = lane < cnt;
   const int p = p0 + (active ? lane : 0);
   const int item = (a.uniform ? k * a.seg_size : __ldg(a.pose_prefix + k)) + p;
+  const int group = chunk * GROUPS_PER_CTA + warp;
 
   // ---- pose of this lane (PLAIN: given; LS: proposal around X[j], R16)
   float4 q, t;
@@ -75,8 +167,7 @@ __global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const Sco
   }
 
   // ---- rotation (homogeneous form, R11) and transformed ligand slots
-  float X[K_SLOTS], Y[K_SLOTS], Z[K_SLOTS];
-  float DN[K_SLOTS], AC[K_SLOTS];
+  Acc r;
   {
     const float w = q.x, x = q.y, y = q.z, z = q.w;
     const float s2 = 2.0f / (w * w + x * x + y * y + z * z);
@@ -85,21 +176,19 @@ __global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const Sco
     const float r20 = s2 * (x * z - w * y), r21 = s2 * (y * z + w * x), r22 = 1.0f - s2 * (x * x + y * y);
     const float4 sh = __ldg(a.shift + spot);
     const float ox = sh.x + t.x, oy = sh.y + t.y, oz = sh.z + t.z;
-    const LigSlot* L = a.lig + (size_t)(chunk * GROUPS_PER_CTA + warp) * K_SLOTS;
+    const LigSlot* L = a.lig + (size_t)group * K_SLOTS;
 #pragma unroll
-    for (int s = 0; s < K_SLOTS; ++s) {
-      const float4 l = __ldg(&L[s].lq);
-      const float4 pp = __ldg(&L[s].p);
-      X[s] = ox + (r00 * l.x + r01 * l.y + r02 * l.z);
-      Y[s] = oy + (r10 * l.x + r11 * l.y + r12 * l.z);
-      Z[s] = oz + (r20 * l.x + r21 * l.y + r22 * l.z);
-      DN[s] = pp.z;
-      AC[s] = pp.w;
+    for (int pp = 0; pp < K_PAIRS; ++pp) {
+      const float4 l0 = __ldg(&L[2 * pp].lq), l1 = __ldg(&L[2 * pp + 1].lq);
+      const float4 p0v = __ldg(&L[2 * pp].p), p1v = __ldg(&L[2 * pp + 1].p);
+      r.X[pp] = make_float2(ox + (r00 * l0.x + r01 * l0.y + r02 * l0.z), ox + (r00 * l1.x + r01 * l1.y + r02 * l1.z));
+      r.Y[pp] = make_float2(oy + (r10 * l0.x + r11 * l0.y + r12 * l0.z), oy + (r10 * l1.x + r11 * l1.y + r12 * l1.z));
+      r.Z[pp] = make_float2(oz + (r20 * l0.x + r21 * l0.y + r22 * l0.z), oz + (r20 * l1.x + r21 * l1.y + r22 * l1.z));
+      r.DN[pp] = make_float2(p0v.z, p1v.z);
+      r.AC[pp] = make_float2(p0v.w, p1v.w);
+      r.Q[pp] = r.A[pp] = r.B[pp] = r.H6[pp] = r.H5[pp] = make_float2(0.0f, 0.0f);
     }
   }
-  float Q[K_SLOTS], A[K_SLOTS], B[K_SLOTS], H6[K_SLOTS], H5[K_SLOTS];
-#pragma unroll
-  for (int s = 0; s < K_SLOTS; ++s) Q[s] = A[s] = B[s] = H6[s] = H5[s] = 0.0f;
 
   // ---- receptor list of the spot through the bulk-copy ring
   const int off = __ldg(a.list_off + spot), len = __ldg(a.list_len + spot);
@@ -117,60 +206,33 @@ __global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const Sco
       bulk_g2s(tile[s], src + (size_t)s * TILE, bytes, &full[s]);
     }
   }
-  const float r2min = a.r2min, rc2 = a.rc2, inv_rc2 = a.inv_rc2;
-  for (int it = 0; it < nt; ++it) {
-    const int st = it % NSTAGE;
-    mbar_wait(&full[st], (uint32_t)(it / NSTAGE) & 1u);
-    const int nvalid = min(TILE, len - it * TILE);
-    const RecAtom* T = tile[st];
-#pragma unroll 1
-    for (int r = 0; r < nvalid; ++r) {
-      const float4 xq = T[r].xq;
-      const float4 pp = T[r].p;
-#pragma unroll
-      for (int s = 0; s < K_SLOTS; ++s) {
-        const float dx = X[s] - xq.x, dy = Y[s] - xq.y, dz = Z[s] - xq.z;
-        float r2 = fmaf(dx, dx, fmaf(dy, dy, dz * dz));
-        r2 = fmaxf(r2, r2min);                                   // R7
-        float sh = 1.0f;
-        if (CUT) {
-          sh = fmaf(r2, -inv_rc2, 1.0f);                         // 1 - r2/rc2 (R6)
-          r2 = (r2 < rc2) ? r2 : __int_as_float(0x7f800000);     // beyond rc: 1/r2 -> 0
-        }
-        const float inv = rcp_approx(r2);
-        float es = (DIEL == 0) ? inv : rsqrt_approx(r2);
-        if (CUT) es = (es * sh) * sh;
-        Q[s] = fmaf(xq.w, es, Q[s]);
-        const float inv2 = inv * inv, inv3 = inv2 * inv, inv6 = inv3 * inv3, inv5 = inv3 * inv2;
-        A[s] = fmaf(pp.x, inv6, A[s]);
-        B[s] = fmaf(pp.y, inv3, B[s]);
-        const float w = fmaf(DN[s], pp.w, AC[s] * pp.z);           // donor_i acc_j + acc_i donor_j (R5)
-        H6[s] = fmaf(w, inv6, H6[s]);
-        H5[s] = fmaf(w, inv5, H5[s]);
-      }
-    }
-    __syncthreads();  // every warp is done with stage st
-    if (threadIdx.x == 0 && it + NSTAGE < nt) {
-      const int nx = it + NSTAGE;
-      const uint32_t bytes = (uint32_t)min(TILE, len - nx * TILE) * (uint32_t)sizeof(RecAtom);
-      mbar_arrive_expect_tx(&full[st], bytes);
-      bulk_g2s(tile[st], src + (size_t)nx * TILE, bytes, &full[st]);
-    }
+  // warp-uniform number of H-bond pairs in this warp's group
+  const int h = min(K_PAIRS, max(0, (group + 1) * K_PAIRS - a.hb_start));
+  switch (h) {
+    case 0: sweep<0, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
+    case 1: sweep<1, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
+    case 2: sweep<2, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
+    case 3: sweep<3, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
+    default: sweep<4, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
   }
 
   // ---- per-slot energies (fp64 combination of the fp32 sums: the terms cancel), fixed-order reduction
   double e = 0.0;
   {
-    const LigSlot* L = a.lig + (size_t)(chunk * GROUPS_PER_CTA + warp) * K_SLOTS;
+    const LigSlot* L = a.lig + (size_t)group * K_SLOTS;
 #pragma unroll
     for (int s = 0; s < K_SLOTS; ++s) {
       const float4 l = __ldg(&L[s].lq);
-      const float4 pp = __ldg(&L[s].p);
-      double es = (double)l.w * (double)Q[s];
-      es = fma((double)pp.x, (double)A[s], es);
-      es = fma(-(double)pp.y, (double)B[s], es);
-      es = fma((double)a.hbC, (double)H6[s], es);
-      es = fma(-(double)a.hbD, (double)H5[s], es);
+      const float4 pv = __ldg(&L[s].p);
+      const int pp = s >> 1;
+      const bool hi = s & 1;
+      double es = (double)l.w * (double)(hi ? r.Q[pp].y : r.Q[pp].x);
+      es = fma((double)pv.x, (double)(hi ? r.A[pp].y : r.A[pp].x), es);
+      es = fma(-(double)pv.y, (double)(hi ? r.B[pp].y : r.B[pp].x), es);
+      if (pv.z + pv.w != 0.0f) {  // H-bond-capable slot (dummies and non-polar atoms: none)
+        es = fma((double)a.hbC, (double)(hi ? r.H6[pp].y : r.H6[pp].x), es);
+        es = fma(-(double)a.hbD, (double)(hi ? r.H5[pp].y : r.H5[pp].x), es);
+      }
       e += es;
     }
   }
@@ -188,10 +250,10 @@ __global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const Sco
         a.poses[pidx].t.w = score;
         if (a.orig) a.score_out[__ldg(a.orig + pidx)] = score;
       } else if (score < old_score) {                            // strict improvement (R16)
-        PoseRec r;
-        r.q = q;
-        r.t = make_float4(t.x, t.y, t.z, score);
-        a.poses[jx] = r;
+        PoseRec rr;
+        rr.q = q;
+        rr.t = make_float4(t.x, t.y, t.z, score);
+        a.poses[jx] = rr;
       }
     }
     if (lane == 0 && chunk == 0 && a.counters) {
