@@ -80,7 +80,7 @@ struct vs_ctx {
   bool all_pairs = false;
   int dielectric = 0;
   float T = 3.0f, rc = 0.0f, rc2 = INFINITY, inv_rc2 = 0.0f, r2min = 0.01f, hbC = 0.0f, hbD = 0.0f;
-  int n_groups = 0, n_chunks = 1, hb_start = 0;
+  int n_groups = 0, n_chunks = 1, hb_base = 0, hb_extra = 0;
   std::vector<int> h_list_len;
   int64_t list_total = 0;
   RecAtom* d_lists = nullptr;
@@ -148,7 +148,8 @@ ScoreArgs base_args(vs_ctx* c) {
   a.shift = c->d_shift;
   a.lig = c->d_lig;
   a.n_groups = c->n_groups;
-  a.hb_start = c->hb_start;
+  a.hb_base = c->hb_base;
+  a.hb_extra = c->hb_extra;
   a.n_chunks = c->n_chunks;
   a.n_lig = c->n_lig;
   a.r2min = c->r2min;
@@ -488,18 +489,19 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     for (int i = 0; i < n_lig; ++i) s += lig_xyz[3 * i + a];
     cen[a] = (float)(s / n_lig);
   }
-  // slot order: atoms without an H-bond role first, then donors/acceptors, as
-  // float2 slot pairs; padding pairs (all-zero dummy atoms, exactly 0 energy) sit in between so
-  // that every H-bond pair is in the tail of the slot sequence (hb_start).
+  // slot layout: each group of K_SLOTS = K_PAIRS float2 slot pairs holds its
+  // H-bond-capable atoms (donors / acceptors) in its last pairs; H-bond pairs are spread evenly
+  // over the groups so that the warps of a CTA carry equal work.  Padding slots are all-zero dummy
+  // atoms (exactly zero energy).
   std::vector<int> plain, hbat;
   for (int i = 0; i < n_lig; ++i) (don[lig_type[i]] != 0.0f || acc[lig_type[i]] != 0.0f ? hbat : plain).push_back(i);
   const int pairs_plain = ((int)plain.size() + 1) / 2, pairs_hb = ((int)hbat.size() + 1) / 2;
   const int groups = (pairs_plain + pairs_hb + K_PAIRS - 1) / K_PAIRS;
   c->n_chunks = (groups + GROUPS_PER_CTA - 1) / GROUPS_PER_CTA;
   c->n_groups = c->n_chunks > 1 ? c->n_chunks * GROUPS_PER_CTA : groups;
-  const int pairs_tot = c->n_groups * K_PAIRS;
-  c->hb_start = pairs_tot - pairs_hb;
-  std::vector<LigSlot> slots((size_t)pairs_tot * 2);
+  c->hb_base = pairs_hb / c->n_groups;
+  c->hb_extra = pairs_hb % c->n_groups;
+  std::vector<LigSlot> slots((size_t)c->n_groups * K_SLOTS);
   std::memset(slots.data(), 0, sizeof(LigSlot) * slots.size());
   double rmax = 0.0;
   auto put = [&](int slot, int i) {
@@ -514,8 +516,25 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     s.p = make_float4(c12[t], c6[t], don[t], acc[t]);
     rmax = std::max(rmax, std::sqrt((double)s.lq.x * s.lq.x + (double)s.lq.y * s.lq.y + (double)s.lq.z * s.lq.z));
   };
-  for (size_t a = 0; a < plain.size(); ++a) put((int)a, plain[a]);
-  for (size_t a = 0; a < hbat.size(); ++a) put(2 * c->hb_start + (int)a, hbat[a]);
+  {
+    size_t ip = 0, ih = 0;
+    for (int g = 0; g < c->n_groups; ++g) {
+      const int h = c->hb_base + (g < c->hb_extra ? 1 : 0);
+      for (int p = 0; p < K_PAIRS; ++p)
+        for (int half = 0; half < 2; ++half) {
+          const int slot = (g * K_PAIRS + p) * 2 + half;
+          if (p < K_PAIRS - h) {
+            if (ip < plain.size()) put(slot, plain[ip++]);
+          } else if (ih < hbat.size()) {
+            put(slot, hbat[ih++]);
+          }
+        }
+    }
+    if (ip != plain.size() || ih != hbat.size()) {
+      vs_destroy(c);
+      return set_err(VS_ERR_INVALID_ARGUMENT, "internal: ligand slot layout");
+    }
+  }
   CKC(cudaMalloc(&c->d_lig, sizeof(LigSlot) * slots.size()), "alloc ligand");
   CKC(cudaMemcpy(c->d_lig, slots.data(), sizeof(LigSlot) * slots.size(), cudaMemcpyHostToDevice), "H2D ligand");
 

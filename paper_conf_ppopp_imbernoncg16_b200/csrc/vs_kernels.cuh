@@ -26,7 +26,7 @@ struct ScoreArgs {
   const float4* shift;       // added to t + R l (all-pairs: c_s - c0; cutoff: 0)
   const LigSlot* lig;
   int n_groups;              // ligand groups of K_SLOTS slots
-  int hb_start;              // first slot pair with hydrogen-bond atoms (pairs before it: no HB)
+  int hb_base, hb_extra;     // group g holds hb_base + (g < hb_extra) H-bond slot pairs, at its end
   int n_chunks;              // ceil(n_groups / GROUPS_PER_CTA)
   int n_lig;                 // real ligand atoms (pair accounting)
   float r2min, rc2, inv_rc2; // rc2 = +inf in all-pairs mode

@@ -23,6 +23,15 @@
 // fp64 in a fixed order (deterministic: identical poses -> identical scores).
 #include "vs_kernels.cuh"
 
+#ifndef VS_UNROLL
+#define VS_UNROLL 2
+#endif
+#ifndef VS_MINB
+#define VS_MINB 2
+#endif
+#define VS_STR2(x) #x
+#define VS_STR(x) VS_STR2(x)
+
 namespace vsk {
 
 __device__ __forceinline__ void locate(const ScoreArgs& a, int bx, int& k, int& blk) {
@@ -42,39 +51,58 @@ __device__ __forceinline__ void locate(const ScoreArgs& a, int bx, int& k, int& 
 
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
 
-struct Acc {
-  float2 X[K_PAIRS], Y[K_PAIRS], Z[K_PAIRS];
-  float2 Q[K_PAIRS], A[K_PAIRS], B[K_PAIRS];
-  float2 H6[K_PAIRS], H5[K_PAIRS];
-  float2 DN[K_PAIRS], AC[K_PAIRS];
-};
-
-// Sweep of the spot's receptor list for one warp whose group has H H-bond pairs.
+// The sweep of one warp over the spot's receptor list.  The group has H slot
+// pairs with H-bond-capable atoms (warp-uniform, compile-time here): the first
+// K_PAIRS - H pairs skip the H-bond arithmetic and keep no H-bond registers.
+// Warps are decoupled: a warp releases a ring stage when it is done with it and
+// the last warp to release a stage refills it (bulk copy), so a warp never
+// waits for the others except on data that has not yet landed.
 template <int H, bool CUT, int DIEL>
-__device__ __forceinline__ void sweep(Acc& r, RecAtom (*tile)[TILE], uint64_t* full, const RecAtom* src, int len,
-                                      int nt, float r2min, float rc2, float inv_rc2) {
+__device__ __forceinline__ double sweep(const ScoreArgs& a, const LigSlot* L, const float (&R)[9], float ox, float oy,
+                                        float oz, RecAtom (*tile)[TILE], uint64_t* full, int* relcnt,
+                                        const RecAtom* src, int len, int nt, int nwarps) {
+  constexpr int HP = H > 0 ? H : 1;
+  constexpr int P0 = K_PAIRS - H;  // first H-bond pair
+  float2 X[K_PAIRS], Y[K_PAIRS], Z[K_PAIRS], Q[K_PAIRS], A[K_PAIRS], B[K_PAIRS];
+  float2 H6[HP], H5[HP];
+  bool DN[2 * HP];
+#pragma unroll
+  for (int p = 0; p < K_PAIRS; ++p) {
+    const float4 l0 = __ldg(&L[2 * p].lq), l1 = __ldg(&L[2 * p + 1].lq);
+    X[p] = make_float2(ox + (R[0] * l0.x + R[1] * l0.y + R[2] * l0.z), ox + (R[0] * l1.x + R[1] * l1.y + R[2] * l1.z));
+    Y[p] = make_float2(oy + (R[3] * l0.x + R[4] * l0.y + R[5] * l0.z), oy + (R[3] * l1.x + R[4] * l1.y + R[5] * l1.z));
+    Z[p] = make_float2(oz + (R[6] * l0.x + R[7] * l0.y + R[8] * l0.z), oz + (R[6] * l1.x + R[7] * l1.y + R[8] * l1.z));
+    Q[p] = A[p] = B[p] = make_float2(0.0f, 0.0f);
+    if (p >= P0) {
+      H6[p - P0] = H5[p - P0] = make_float2(0.0f, 0.0f);
+      DN[2 * (p - P0)] = __ldg(&L[2 * p].p.z) != 0.0f;
+      DN[2 * (p - P0) + 1] = __ldg(&L[2 * p + 1].p.z) != 0.0f;
+    }
+  }
+  const float r2min = a.r2min, rc2 = a.rc2, inv_rc2 = a.inv_rc2;
   const float INF = __int_as_float(0x7f800000);
+  const int lane = threadIdx.x & 31;
   for (int it = 0; it < nt; ++it) {
     const int st = it % NSTAGE;
     mbar_wait(&full[st], (uint32_t)(it / NSTAGE) & 1u);
     const int nvalid = min(TILE, len - it * TILE);
     const RecAtom* T = tile[st];
-#pragma unroll 2
+    _Pragma(VS_STR(unroll VS_UNROLL))
     for (int j = 0; j < nvalid; ++j) {
       const float4 xq = T[j].xq;
       const float4 pp = T[j].p;
 #pragma unroll
       for (int p = 0; p < K_PAIRS; ++p) {
-        const float2 dx = __fadd2_rn(r.X[p], f2(-xq.x));
-        const float2 dy = __fadd2_rn(r.Y[p], f2(-xq.y));
-        const float2 dz = __fadd2_rn(r.Z[p], f2(-xq.z));
+        const float2 dx = __fadd2_rn(X[p], f2(-xq.x));
+        const float2 dy = __fadd2_rn(Y[p], f2(-xq.y));
+        const float2 dz = __fadd2_rn(Z[p], f2(-xq.z));
         float2 r2 = __fmul2_rn(dx, dx);
         r2 = __ffma2_rn(dy, dy, r2);
         r2 = __ffma2_rn(dz, dz, r2);
         r2.x = fmaxf(r2.x, r2min);                                   // R7
         r2.y = fmaxf(r2.y, r2min);
         bool inx = true, iny = true;
-        float2 r2u = r2;
+        const float2 r2u = r2;
         if (CUT) {
           inx = r2.x < rc2;
           iny = r2.y < rc2;
@@ -100,35 +128,65 @@ __device__ __forceinline__ void sweep(Acc& r, RecAtom (*tile)[TILE], uint64_t* f
             es = __fmul2_rn(__fmul2_rn(es, sh), sh);
           }
         }
-        r.Q[p] = __ffma2_rn(es, f2(xq.w), r.Q[p]);
+        Q[p] = __ffma2_rn(es, f2(xq.w), Q[p]);
         const float2 inv2 = __fmul2_rn(inv, inv);
         const float2 inv3 = __fmul2_rn(inv2, inv);
         const float2 inv6 = __fmul2_rn(inv3, inv3);
-        r.A[p] = __ffma2_rn(inv6, f2(pp.x), r.A[p]);
-        r.B[p] = __ffma2_rn(inv3, f2(pp.y), r.B[p]);
-        if (p >= K_PAIRS - H) {                                      // compile-time after unrolling
+        A[p] = __ffma2_rn(inv6, f2(pp.x), A[p]);
+        B[p] = __ffma2_rn(inv3, f2(pp.y), B[p]);
+        if (p >= P0) {                                               // compile-time after unrolling
+          const int hq = p - P0;
           const float2 inv5 = __fmul2_rn(inv3, inv2);
-          // donor slot pairs with receptor acceptors, acceptor slot with receptor donors (R5)
-          const float2 w = make_float2(r.DN[p].x != 0.0f ? pp.w : pp.z, r.DN[p].y != 0.0f ? pp.w : pp.z);
-          r.H6[p] = __ffma2_rn(w, inv6, r.H6[p]);
-          r.H5[p] = __ffma2_rn(w, inv5, r.H5[p]);
+          // a donor slot bonds with receptor acceptors, an acceptor slot with receptor donors (R5)
+          const float2 w = make_float2(DN[2 * hq] ? pp.w : pp.z, DN[2 * hq + 1] ? pp.w : pp.z);
+          H6[hq] = __ffma2_rn(w, inv6, H6[hq]);
+          H5[hq] = __ffma2_rn(w, inv5, H5[hq]);
         }
       }
     }
-    __syncthreads();  // every warp is done with stage st
-    if (threadIdx.x == 0 && it + NSTAGE < nt) {
-      const int nx = it + NSTAGE;
-      const uint32_t bytes = (uint32_t)min(TILE, len - nx * TILE) * (uint32_t)sizeof(RecAtom);
-      mbar_arrive_expect_tx(&full[st], bytes);
-      bulk_g2s(tile[st], src + (size_t)nx * TILE, bytes, &full[st]);
+    // release stage st; the last warp to release it refills it with tile it + NSTAGE
+    __syncwarp();
+    if (lane == 0) {
+      __threadfence_block();
+      if (atomicAdd(&relcnt[st], 1) == nwarps - 1) {
+        atomicExch(&relcnt[st], 0);
+        if (it + NSTAGE < nt) {
+          const int nx = it + NSTAGE;
+          const uint32_t bytes = (uint32_t)min(TILE, len - nx * TILE) * (uint32_t)sizeof(RecAtom);
+          fence_proxy_async();
+          mbar_arrive_expect_tx(&full[st], bytes);
+          bulk_g2s(tile[st], src + (size_t)nx * TILE, bytes, &full[st]);
+        }
+      }
     }
   }
+  // per-slot energies: fp64 combination of the fp32 sums (the terms cancel)
+  double e = 0.0;
+#pragma unroll
+  for (int s = 0; s < K_SLOTS; ++s) {
+    const int p = s >> 1;
+    const bool hi = s & 1;
+    const float4 l = __ldg(&L[s].lq);
+    const float4 pv = __ldg(&L[s].p);
+    double es = (double)l.w * (double)(hi ? Q[p].y : Q[p].x);
+    es = fma((double)pv.x, (double)(hi ? A[p].y : A[p].x), es);
+    es = fma(-(double)pv.y, (double)(hi ? B[p].y : B[p].x), es);
+    if (p >= P0) {
+      const int hq = p - P0;
+      const double hsel = (double)(pv.z + pv.w);  // 1 for donors / acceptors, 0 for padding atoms
+      es = fma(hsel * a.hbC, (double)(hi ? H6[hq].y : H6[hq].x), es);
+      es = fma(-hsel * a.hbD, (double)(hi ? H5[hq].y : H5[hq].x), es);
+    }
+    e += es;
+  }
+  return e;
 }
 
 template <int MODE, bool CUT, int DIEL>
-__global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const ScoreArgs a) {
+__global__ void __launch_bounds__(GROUPS_PER_CTA * 32, VS_MINB) score_kernel(const ScoreArgs a) {
   __shared__ __align__(128) RecAtom tile[NSTAGE][TILE];
   __shared__ __align__(8) uint64_t full[NSTAGE];
+  __shared__ int relcnt[NSTAGE];
   __shared__ double red[GROUPS_PER_CTA][32];
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -166,36 +224,31 @@ __global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const Sco
             2u * (uint32_t)a.l);
   }
 
-  // ---- rotation (homogeneous form, R11) and transformed ligand slots
-  Acc r;
+  // ---- rotation (homogeneous form, R11)
+  float R[9];
+  float ox, oy, oz;
   {
     const float w = q.x, x = q.y, y = q.z, z = q.w;
     const float s2 = 2.0f / (w * w + x * x + y * y + z * z);
-    const float r00 = 1.0f - s2 * (y * y + z * z), r01 = s2 * (x * y - w * z), r02 = s2 * (x * z + w * y);
-    const float r10 = s2 * (x * y + w * z), r11 = 1.0f - s2 * (x * x + z * z), r12 = s2 * (y * z - w * x);
-    const float r20 = s2 * (x * z - w * y), r21 = s2 * (y * z + w * x), r22 = 1.0f - s2 * (x * x + y * y);
+    R[0] = 1.0f - s2 * (y * y + z * z); R[1] = s2 * (x * y - w * z); R[2] = s2 * (x * z + w * y);
+    R[3] = s2 * (x * y + w * z); R[4] = 1.0f - s2 * (x * x + z * z); R[5] = s2 * (y * z - w * x);
+    R[6] = s2 * (x * z - w * y); R[7] = s2 * (y * z + w * x); R[8] = 1.0f - s2 * (x * x + y * y);
     const float4 sh = __ldg(a.shift + spot);
-    const float ox = sh.x + t.x, oy = sh.y + t.y, oz = sh.z + t.z;
-    const LigSlot* L = a.lig + (size_t)group * K_SLOTS;
-#pragma unroll
-    for (int pp = 0; pp < K_PAIRS; ++pp) {
-      const float4 l0 = __ldg(&L[2 * pp].lq), l1 = __ldg(&L[2 * pp + 1].lq);
-      const float4 p0v = __ldg(&L[2 * pp].p), p1v = __ldg(&L[2 * pp + 1].p);
-      r.X[pp] = make_float2(ox + (r00 * l0.x + r01 * l0.y + r02 * l0.z), ox + (r00 * l1.x + r01 * l1.y + r02 * l1.z));
-      r.Y[pp] = make_float2(oy + (r10 * l0.x + r11 * l0.y + r12 * l0.z), oy + (r10 * l1.x + r11 * l1.y + r12 * l1.z));
-      r.Z[pp] = make_float2(oz + (r20 * l0.x + r21 * l0.y + r22 * l0.z), oz + (r20 * l1.x + r21 * l1.y + r22 * l1.z));
-      r.DN[pp] = make_float2(p0v.z, p1v.z);
-      r.AC[pp] = make_float2(p0v.w, p1v.w);
-      r.Q[pp] = r.A[pp] = r.B[pp] = r.H6[pp] = r.H5[pp] = make_float2(0.0f, 0.0f);
-    }
+    ox = sh.x + t.x;
+    oy = sh.y + t.y;
+    oz = sh.z + t.z;
   }
+  const LigSlot* L = a.lig + (size_t)group * K_SLOTS;
 
   // ---- receptor list of the spot through the bulk-copy ring
   const int off = __ldg(a.list_off + spot), len = __ldg(a.list_len + spot);
   const RecAtom* src = a.lists + off;
   const int nt = (len + TILE - 1) / TILE;
   if (threadIdx.x == 0) {
-    for (int s = 0; s < NSTAGE; ++s) mbar_init(&full[s], 1);
+    for (int s = 0; s < NSTAGE; ++s) {
+      mbar_init(&full[s], 1);
+      relcnt[s] = 0;
+    }
     fence_mbar_init();
   }
   __syncthreads();
@@ -206,36 +259,17 @@ __global__ void __launch_bounds__(GROUPS_PER_CTA * 32, 2) score_kernel(const Sco
       bulk_g2s(tile[s], src + (size_t)s * TILE, bytes, &full[s]);
     }
   }
-  // warp-uniform number of H-bond pairs in this warp's group
-  const int h = min(K_PAIRS, max(0, (group + 1) * K_PAIRS - a.hb_start));
+  // warp-uniform number of H-bond pairs in this warp's group (spread evenly over the groups)
+  const int h = a.hb_base + (group < a.hb_extra ? 1 : 0);
+  double e;
   switch (h) {
-    case 0: sweep<0, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
-    case 1: sweep<1, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
-    case 2: sweep<2, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
-    case 3: sweep<3, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
-    default: sweep<4, CUT, DIEL>(r, tile, full, src, len, nt, a.r2min, a.rc2, a.inv_rc2); break;
+    case 0: e = sweep<0, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
+    case 1: e = sweep<1, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
+    case 2: e = sweep<2, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
+    case 3: e = sweep<3, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
+    default: e = sweep<4, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
   }
 
-  // ---- per-slot energies (fp64 combination of the fp32 sums: the terms cancel), fixed-order reduction
-  double e = 0.0;
-  {
-    const LigSlot* L = a.lig + (size_t)group * K_SLOTS;
-#pragma unroll
-    for (int s = 0; s < K_SLOTS; ++s) {
-      const float4 l = __ldg(&L[s].lq);
-      const float4 pv = __ldg(&L[s].p);
-      const int pp = s >> 1;
-      const bool hi = s & 1;
-      double es = (double)l.w * (double)(hi ? r.Q[pp].y : r.Q[pp].x);
-      es = fma((double)pv.x, (double)(hi ? r.A[pp].y : r.A[pp].x), es);
-      es = fma(-(double)pv.y, (double)(hi ? r.B[pp].y : r.B[pp].x), es);
-      if (pv.z + pv.w != 0.0f) {  // H-bond-capable slot (dummies and non-polar atoms: none)
-        es = fma((double)a.hbC, (double)(hi ? r.H6[pp].y : r.H6[pp].x), es);
-        es = fma(-(double)a.hbD, (double)(hi ? r.H5[pp].y : r.H5[pp].x), es);
-      }
-      e += es;
-    }
-  }
   red[warp][lane] = e;
   __syncthreads();
   if (warp == 0) {

@@ -58,7 +58,7 @@ _lib = None
 
 
 def library_path() -> str:
-    return _build.LIB
+    return os.environ.get("VS_LIB") or _build.LIB
 
 
 def load(build_if_stale: bool = True):
@@ -66,7 +66,9 @@ def load(build_if_stale: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    path = _build.LIB
+    path = os.environ.get("VS_LIB") or _build.LIB
+    if os.environ.get("VS_LIB"):
+        build_if_stale = False
     if build_if_stale:
         try:
             path = _build.build()
