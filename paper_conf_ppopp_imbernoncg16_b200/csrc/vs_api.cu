@@ -63,6 +63,8 @@ struct DevBuf {
   }
 };
 
+constexpr int NSUB = 4;  // spot groups (streams) of one vs_run
+
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
            B_SORTED, B_ORIG, B_BEST, B_BESTS, B_COUNT };
 
@@ -91,6 +93,8 @@ struct vs_ctx {
   int* d_iota = nullptr;
   unsigned long long* d_counters = nullptr;
   cudaStream_t stream = nullptr;
+  cudaStream_t sub[NSUB] = {};          // per-spot-group streams of vs_run
+  cudaEvent_t ev_fork = nullptr, ev_join[NSUB] = {};
   DevBuf buf[B_COUNT];
   bool poisoned = false;
   // instrumentation
@@ -226,6 +230,76 @@ vs_status trace_idx(vs_ctx* c, Tracer* tr, cudaStream_t st, int stage, int g, in
   return VS_OK;
 }
 
+// One group of spots running Algorithm 1 on its own stream.
+struct Group {
+  int ns = 0;
+  const int* seg = nullptr;
+  PoseRec *S = nullptr, *S2 = nullptr, *C = nullptr;
+  int* J = nullptr;
+  cudaStream_t st = nullptr;
+  ScoreArgs plain, ls;
+  int plain_blocks = 0, ls_blocks = 0;
+  bool in_b = false;  // the current population S sits in the second (B) buffer
+};
+
+// Improve (R16-R17): the best m of X by (score, index), then L fused
+// perturb -> score -> accept launches.
+vs_status improve_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, PoseRec* X, int g, Tracer* tr) {
+  const int P = mp->population;
+  CK(launch_popsort(0, X, nullptr, nullptr, q.J, q.ns, P, m, q.st), "select launch");
+  c->launches++;
+  vs_status r = trace_idx(c, tr, q.st, VS_TRACE_SELECT, g, q.ns, m, q.J);
+  if (r != VS_OK) return r;
+  for (int l = 0; l < mp->ls_steps; ++l) {
+    ScoreArgs a = q.ls;
+    a.poses = X;
+    a.g = g;
+    a.l = l;
+    if ((r = score_launch(c, a, MODE_LS, q.ls_blocks, q.st)) != VS_OK) return r;
+    if ((r = trace_poses(c, tr, q.st, VS_TRACE_LS, g, l, q.ns, P, X)) != VS_OK) return r;
+  }
+  return VS_OK;
+}
+
+// Initialize(S): random population, scored, improved when f > 0, sorted.
+vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, uint64_t seed, int m, Tracer* tr) {
+  const int P = mp->population;
+  CK(launch_init(q.S, q.ns, P, q.seg, seed, c->T, q.st), "init launch");
+  c->launches++;
+  vs_status r = trace_poses(c, tr, q.st, VS_TRACE_INIT, 0, 0, q.ns, P, q.S);
+  if (r != VS_OK) return r;
+  ScoreArgs a = q.plain;
+  a.poses = q.S;
+  if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
+  if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, 0, 0, q.ns, P, q.S)) != VS_OK) return r;
+  if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.S, 0, tr)) != VS_OK) return r;
+  CK(launch_popsort(1, q.S, nullptr, q.S2, nullptr, q.ns, P, m, q.st), "sort launch");
+  c->launches++;
+  std::swap(q.S, q.S2);
+  q.in_b = !q.in_b;
+  return trace_poses(c, tr, q.st, VS_TRACE_SORTED, 0, 0, q.ns, P, q.S);
+}
+
+// One pass of the while-loop body: Select + Combine, score, Improve, Include.
+vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, uint64_t seed, int m, int g, Tracer* tr) {
+  const int P = mp->population;
+  CK(launch_combine(q.S, q.C, q.ns, P, q.seg, seed, g, mp->p_mut, mp->mut_trans, mp->mut_rot, c->T, q.st),
+     "combine launch");
+  c->launches++;
+  vs_status r = trace_poses(c, tr, q.st, VS_TRACE_COMBINED, g, 0, q.ns, P, q.C);
+  if (r != VS_OK) return r;
+  ScoreArgs a = q.plain;
+  a.poses = q.C;
+  if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
+  if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, g, 0, q.ns, P, q.C)) != VS_OK) return r;
+  if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.C, g, tr)) != VS_OK) return r;
+  CK(launch_popsort(2, q.S, q.C, q.S2, nullptr, q.ns, P, m, q.st), "include launch");
+  c->launches++;
+  std::swap(q.S, q.S2);
+  q.in_b = !q.in_b;
+  return trace_poses(c, tr, q.st, VS_TRACE_INCLUDED, g, 0, q.ns, P, q.S);
+}
+
 // The generation loop (Algorithm 1) for n_sel spots, all on stream st.
 vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
                    float* d_best_pose, float* d_best_score, cudaStream_t st, Tracer* tr) {
@@ -241,7 +315,6 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
       if (spot_ids[k] < 0 || spot_ids[k] >= c->n_spots) return set_err(VS_ERR_INVALID_ARGUMENT, "spot id out of range");
   const int P = mp->population;
   const int m = improve_count(mp);
-  const bool improve = mp->improve_frac > 0.0f;
   const size_t pop_bytes = sizeof(PoseRec) * (size_t)ns * P;
   CK(c->buf[B_SEG].ensure(sizeof(int) * ns), "alloc");
   CK(c->buf[B_SA].ensure(pop_bytes), "alloc");
@@ -254,80 +327,62 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     CK(cudaMemcpyAsync(seg, spot_ids, sizeof(int) * ns, cudaMemcpyHostToDevice, st), "H2D spot ids");
   else
     CK(cudaMemcpyAsync(seg, c->d_iota, sizeof(int) * ns, cudaMemcpyDeviceToDevice, st), "D2D spot ids");
-  PoseRec* S = (PoseRec*)c->buf[B_SA].p;
-  PoseRec* S2 = (PoseRec*)c->buf[B_SB].p;
-  PoseRec* C = (PoseRec*)c->buf[B_C].p;
-  int* J = (int*)c->buf[B_J].p;
+  PoseRec* SA = (PoseRec*)c->buf[B_SA].p;
+  PoseRec* SB = (PoseRec*)c->buf[B_SB].p;
+  PoseRec* CC = (PoseRec*)c->buf[B_C].p;
+  int* JJ = (int*)c->buf[B_J].p;
+  double* part = (double*)c->buf[B_PART].p;
 
-  ScoreArgs plain = base_args(c);
-  plain.nseg = ns;
-  plain.seg_spot = seg;
-  plain.uniform = 1;
-  plain.seg_size = P;
-  plain.bps = (P + POSES_PER_CTA - 1) / POSES_PER_CTA;
-  plain.seg_stride = P;
-  plain.P = P;
-  plain.partial = (double*)c->buf[B_PART].p;
-  ScoreArgs ls = plain;
-  ls.seg_size = m;
-  ls.bps = (m + POSES_PER_CTA - 1) / POSES_PER_CTA;
-  ls.J = J;
-  ls.m = m;
-  ls.seed = seed;
-  ls.ls_trans = mp->ls_trans;
-  ls.ls_rot = mp->ls_rot;
-  const int plain_blocks = ns * plain.bps, ls_blocks = ns * ls.bps;
-
-  auto improve_step = [&](PoseRec* X, int g) -> vs_status {
-    CK(launch_popsort(0, X, nullptr, nullptr, J, ns, P, m, st), "select launch");
-    c->launches++;
-    vs_status r = trace_idx(c, tr, st, VS_TRACE_SELECT, g, ns, m, J);
-    if (r != VS_OK) return r;
-    for (int l = 0; l < mp->ls_steps; ++l) {
-      ScoreArgs a = ls;
-      a.poses = X;
-      a.g = g;
-      a.l = l;
-      r = score_launch(c, a, MODE_LS, ls_blocks, st);
-      if (r != VS_OK) return r;
-      r = trace_poses(c, tr, st, VS_TRACE_LS, g, l, ns, P, X);
-      if (r != VS_OK) return r;
+  // Spots are independent: split them into groups whose generation loops run on separate
+  // streams, enqueued generation by generation, so one group's kernels fill the wave tails of
+  // another's.
+  const int G = tr ? 1 : std::max(1, std::min(NSUB, ns / 64));
+  Group grp[NSUB];
+  CK(cudaEventRecord(c->ev_fork, st), "event record");
+  for (int gi = 0; gi < G; ++gi) {
+    const int k0 = (int)((int64_t)ns * gi / G), k1 = (int)((int64_t)ns * (gi + 1) / G);
+    Group& q = grp[gi];
+    q.ns = k1 - k0;
+    q.seg = seg + k0;
+    q.S = SA + (size_t)k0 * P;
+    q.S2 = SB + (size_t)k0 * P;
+    q.C = CC + (size_t)k0 * P;
+    q.J = JJ + (size_t)k0 * m;
+    q.st = G > 1 ? c->sub[gi] : st;
+    if (G > 1) CK(cudaStreamWaitEvent(q.st, c->ev_fork, 0), "stream wait");
+    ScoreArgs& pl = q.plain;
+    pl = base_args(c);
+    pl.nseg = q.ns;
+    pl.seg_spot = q.seg;
+    pl.uniform = 1;
+    pl.seg_size = P;
+    pl.bps = (P + POSES_PER_CTA - 1) / POSES_PER_CTA;
+    pl.seg_stride = P;
+    pl.P = P;
+    pl.partial = part ? part + (size_t)k0 * P * c->n_chunks : nullptr;
+    q.ls = pl;
+    q.ls.seg_size = m;
+    q.ls.bps = (m + POSES_PER_CTA - 1) / POSES_PER_CTA;
+    q.ls.J = q.J;
+    q.ls.m = m;
+    q.ls.seed = seed;
+    q.ls.ls_trans = mp->ls_trans;
+    q.ls.ls_rot = mp->ls_rot;
+    q.plain_blocks = q.ns * pl.bps;
+    q.ls_blocks = q.ns * q.ls.bps;
+  }
+  vs_status r;
+  for (int gi = 0; gi < G; ++gi)
+    if ((r = gen_initialize(c, grp[gi], mp, seed, m, tr)) != VS_OK) return r;
+  for (int g = 1; g <= mp->generations; ++g)         // End(S): fixed G (R20)
+    for (int gi = 0; gi < G; ++gi)
+      if ((r = gen_step(c, grp[gi], mp, seed, m, g, tr)) != VS_OK) return r;
+  if (G > 1)
+    for (int gi = 0; gi < G; ++gi) {
+      CK(cudaEventRecord(c->ev_join[gi], grp[gi].st), "event record");
+      CK(cudaStreamWaitEvent(st, c->ev_join[gi], 0), "stream wait");
     }
-    return VS_OK;
-  };
-
-  // Initialize(S)
-  CK(launch_init(S, ns, P, seg, seed, c->T, st), "init launch");
-  c->launches++;
-  vs_status r = trace_poses(c, tr, st, VS_TRACE_INIT, 0, 0, ns, P, S);
-  if (r != VS_OK) return r;
-  {
-    ScoreArgs a = plain;
-    a.poses = S;
-    if ((r = score_launch(c, a, MODE_PLAIN, plain_blocks, st)) != VS_OK) return r;
-  }
-  if ((r = trace_poses(c, tr, st, VS_TRACE_SCORED, 0, 0, ns, P, S)) != VS_OK) return r;
-  if (improve && (r = improve_step(S, 0)) != VS_OK) return r;
-  CK(launch_popsort(1, S, nullptr, S2, nullptr, ns, P, m, st), "sort launch");
-  c->launches++;
-  std::swap(S, S2);
-  if ((r = trace_poses(c, tr, st, VS_TRACE_SORTED, 0, 0, ns, P, S)) != VS_OK) return r;
-  // while !End(S): Select, Combine, Improve, Include
-  for (int g = 1; g <= mp->generations; ++g) {
-    CK(launch_combine(S, C, ns, P, seg, seed, g, mp->p_mut, mp->mut_trans, mp->mut_rot, c->T, st), "combine launch");
-    c->launches++;
-    if ((r = trace_poses(c, tr, st, VS_TRACE_COMBINED, g, 0, ns, P, C)) != VS_OK) return r;
-    ScoreArgs a = plain;
-    a.poses = C;
-    if ((r = score_launch(c, a, MODE_PLAIN, plain_blocks, st)) != VS_OK) return r;
-    if ((r = trace_poses(c, tr, st, VS_TRACE_SCORED, g, 0, ns, P, C)) != VS_OK) return r;
-    if (improve && (r = improve_step(C, g)) != VS_OK) return r;
-    CK(launch_popsort(2, S, C, S2, nullptr, ns, P, m, st), "include launch");
-    c->launches++;
-    std::swap(S, S2);
-    if ((r = trace_poses(c, tr, st, VS_TRACE_INCLUDED, g, 0, ns, P, S)) != VS_OK) return r;
-  }
-  CK(launch_best(S, ns, P, d_best_pose, d_best_score, st), "best launch");
+  CK(launch_best(grp[0].in_b ? SB : SA, ns, P, d_best_pose, d_best_score, st), "best launch");
   c->launches++;
   return VS_OK;
 }
@@ -482,6 +537,11 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   } while (0)
 
   CKC(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking), "stream create");
+  for (int i = 0; i < NSUB; ++i) {
+    CKC(cudaStreamCreateWithFlags(&c->sub[i], cudaStreamNonBlocking), "stream create");
+    CKC(cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming), "event create");
+  }
+  CKC(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming), "event create");
   // ligand: centred on the fp32-rounded fp64 centroid (R11); slots in K_SLOTS groups
   float cen[3];
   for (int a = 0; a < 3; ++a) {
@@ -726,6 +786,11 @@ void vs_destroy(vs_ctx* c) {
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (c->stream) cudaStreamDestroy(c->stream);
+  for (int i = 0; i < NSUB; ++i) {
+    if (c->sub[i]) cudaStreamDestroy(c->sub[i]);
+    if (c->ev_join[i]) cudaEventDestroy(c->ev_join[i]);
+  }
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   delete c;
 }
 

@@ -29,6 +29,11 @@
 #ifndef VS_MINB
 #define VS_MINB 2
 #endif
+#ifdef VS_MAXNREG
+#define VS_REGCAP __maxnreg__(VS_MAXNREG)
+#else
+#define VS_REGCAP __launch_bounds__(GROUPS_PER_CTA * 32, VS_MINB)
+#endif
 #define VS_STR2(x) #x
 #define VS_STR(x) VS_STR2(x)
 
@@ -183,7 +188,7 @@ __device__ __forceinline__ double sweep(const ScoreArgs& a, const LigSlot* L, co
 }
 
 template <int MODE, bool CUT, int DIEL>
-__global__ void __launch_bounds__(GROUPS_PER_CTA * 32, VS_MINB) score_kernel(const ScoreArgs a) {
+__global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
   __shared__ __align__(128) RecAtom tile[NSTAGE][TILE];
   __shared__ __align__(8) uint64_t full[NSTAGE];
   __shared__ int relcnt[NSTAGE];
