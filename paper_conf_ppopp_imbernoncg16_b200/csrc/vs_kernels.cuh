@@ -9,7 +9,10 @@ namespace vsk {
 
 constexpr int K_SLOTS = 8;          // ligand atoms per thread (register blocking)
 constexpr int K_PAIRS = K_SLOTS / 2; // slot pairs: one float2 lane-pair per FFMA2
-constexpr int GROUPS_PER_CTA = 8;   // warps (ligand-atom groups) per CTA at most
+#ifndef VS_GPC
+#define VS_GPC 8
+#endif
+constexpr int GROUPS_PER_CTA = VS_GPC;  // warps (ligand-atom groups) per CTA at most
 constexpr int POSES_PER_CTA = 32;   // one pose per lane
 constexpr int TILE = 128;           // receptor atoms per shared-memory stage (4 KB)
 constexpr int NSTAGE = 4;           // bulk-copy ring depth

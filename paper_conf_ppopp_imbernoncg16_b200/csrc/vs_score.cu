@@ -27,7 +27,7 @@
 #define VS_UNROLL 2
 #endif
 #ifndef VS_MINB
-#define VS_MINB 2
+#define VS_MINB (16 / GROUPS_PER_CTA)
 #endif
 #ifdef VS_MAXNREG
 #define VS_REGCAP __maxnreg__(VS_MAXNREG)
