@@ -216,10 +216,18 @@ def main():
     from paper_conf_ppopp_imbernoncg16_b200 import dist as vdist
     from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
 
+    # one process per GPU; VS_BENCH_BACKEND=gloo (CPU collectives, ranks may share a GPU) exercises the
+    # multi-rank path on a single-GPU box
+    backend = os.environ.get("VS_BENCH_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    cdev = dev if backend == "nccl" else torch.device("cpu")   # where collective tensors live
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     prob = synth.make_problem(args.config)
     cfg = prob.cfg
     G = cfg.generations if args.generations is None else args.generations
@@ -259,7 +267,7 @@ def main():
                         work(a, b)
                 rec = torch.cat(parts) if parts else torch.zeros((0, vdist.REC), device=dev)
             if world > 1:
-                vdist.gather_records(rec, dev)
+                vdist.gather_records(rec, cdev)
         return rec
 
     for i in range(args.warmup):
@@ -285,8 +293,8 @@ def main():
     st = ctx.stats()
     ctx.set_timing(False)
     # whole-job totals and max-over-ranks time
-    tot = torch.tensor([st["pairs"], st["poses_scored"], st["kernel_launches"]], dtype=torch.float64, device=dev)
-    tmax = torch.tensor([ms_rank], dtype=torch.float64, device=dev)
+    tot = torch.tensor([st["pairs"], st["poses_scored"], st["kernel_launches"]], dtype=torch.float64, device=cdev)
+    tmax = torch.tensor([ms_rank], dtype=torch.float64, device=cdev)
     if world > 1:
         dist.all_reduce(tot, op=dist.ReduceOp.SUM)
         dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
@@ -329,8 +337,8 @@ def main():
             with vs.Context(*host, sp=sp, device=local) as c2:
                 c2.run(mp, args.seed + rank, None)
                 e2e_ctx_stats.append(c2.stats())
-        dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
-        e2e_pairs = torch.tensor([sum(s["pairs"] for s in e2e_ctx_stats)], dtype=torch.float64, device=dev)
+        dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=cdev)
+        e2e_pairs = torch.tensor([sum(s["pairs"] for s in e2e_ctx_stats)], dtype=torch.float64, device=cdev)
         if world > 1:
             dist.all_reduce(dt, op=dist.ReduceOp.MAX)
             dist.all_reduce(e2e_pairs, op=dist.ReduceOp.SUM)

@@ -7,8 +7,11 @@
 
 namespace vsk {
 
-constexpr int K_SLOTS = 8;          // ligand atoms per thread (register blocking)
-constexpr int K_PAIRS = K_SLOTS / 2; // slot pairs: one float2 lane-pair per FFMA2
+#ifndef VS_KPAIRS
+#define VS_KPAIRS 4
+#endif
+constexpr int K_PAIRS = VS_KPAIRS;   // slot pairs per thread: one float2 lane-pair per FFMA2
+constexpr int K_SLOTS = 2 * K_PAIRS; // ligand atoms per thread (register blocking)
 #ifndef VS_GPC
 #define VS_GPC 8
 #endif

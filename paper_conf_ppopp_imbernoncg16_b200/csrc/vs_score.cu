@@ -268,11 +268,11 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
   const int h = a.hb_base + (group < a.hb_extra ? 1 : 0);
   double e;
   switch (h) {
-    case 0: e = sweep<0, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
-    case 1: e = sweep<1, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
-    case 2: e = sweep<2, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
-    case 3: e = sweep<3, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
-    default: e = sweep<4, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
+#define VS_CASE(HH) \
+  case HH: e = sweep<(HH <= K_PAIRS ? HH : K_PAIRS), CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
+    VS_CASE(0) VS_CASE(1) VS_CASE(2) VS_CASE(3) VS_CASE(4) VS_CASE(5) VS_CASE(6) VS_CASE(7)
+#undef VS_CASE
+    default: e = sweep<K_PAIRS, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
   }
 
   red[warp][lane] = e;
