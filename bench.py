@@ -214,7 +214,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_ppopp_imbernoncg16_b200 import dist as vdist
-    from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
+    from paper_conf_ppopp_imbernoncg16_b200 import screen, synth, vs
 
     # one process per GPU; VS_BENCH_BACKEND=gloo (CPU collectives, ranks may share a GPU) exercises the
     # multi-rank path on a single-GPU box
@@ -234,20 +234,62 @@ def main():
     cutoff = 12.0 if args.mode == "cutoff" else 0.0
     sp = vs.score_params(cutoff=cutoff)
     mp = vs.mh_preset(args.preset, population=cfg.population, generations=G)
-    ctx = vs.Context.from_problem(prob, sp, device=local)
+    sweep = cfg.n_ligands > 1
     n_spots = cfg.n_spots
     stream = torch.cuda.Stream(device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # > 126 MB L2
-    best_pose = torch.empty((n_spots, 7), dtype=torch.float32, device=dev)
-    best_score = torch.empty(n_spots, dtype=torch.float32, device=dev)
-    schedule = vdist.chunk_schedule(n_spots, world, min_chunk=4) if args.scaling == "strong" else None
     store = dist.distributed_c10d._get_default_store() if world > 1 else None
+    if sweep:
+        # screening sweep (N1): units (ligand, spot chunk), largest ligands first, dynamic queue
+        scr = screen.Screen(prob.rec, prob.spots, prob.ligands, sp, mp, args.seed, device=local)
+        sizes = [len(m.q) for m in prob.ligands]
+        units = screen.unit_schedule(sizes, n_spots, world, min_chunk=16)
+        if world == 1:
+            scr.prepare(range(len(prob.ligands)))
+        res_pose = torch.empty((len(prob.ligands), n_spots, 7), dtype=torch.float32, device=dev)
+        res_score = torch.empty((len(prob.ligands), n_spots), dtype=torch.float32, device=dev)
+        ctx = None
+    else:
+        ctx = vs.Context.from_problem(prob, sp, device=local)
+        best_pose = torch.empty((n_spots, 7), dtype=torch.float32, device=dev)
+        best_score = torch.empty(n_spots, dtype=torch.float32, device=dev)
+        schedule = vdist.chunk_schedule(n_spots, world, min_chunk=4) if args.scaling == "strong" else None
+
+    class Work:
+        """stats / timing over every context this rank uses"""
+        def stats(self):
+            return scr.stats() if sweep else ctx.stats()
+
+        def reset_stats(self):
+            scr.reset_stats() if sweep else ctx.reset_stats()
+
+        def set_timing(self, on):
+            for c in (scr.ctx.values() if sweep else [ctx]):
+                c.set_timing(on)
+
+    work_obj = Work()
 
     def step(i: int):
         """One whole-job pass: returns this rank's records (device tensor) for the gather."""
         with torch.cuda.stream(stream):
             flush.zero_()
-            if args.scaling == "weak":
+            if sweep:
+                parts = []
+
+                def unit(k0, k1):
+                    for li, a, b in units[k0:k1]:
+                        scr.run_unit(li, a, b, res_pose[li, a:b], res_score[li, a:b], stream)
+                        ids = torch.arange(a, b, dtype=torch.float32, device=dev)
+                        lid = torch.full_like(ids, float(li))
+                        parts.append(torch.cat([lid[:, None], ids[:, None], res_score[li, a:b, None],
+                                                res_pose[li, a:b]], 1))
+
+                if world > 1:
+                    vdist.claim_chunks(store, f"s{i}", [(k, k + 1) for k in range(len(units))], unit)
+                else:
+                    unit(0, len(units))
+                rec = torch.cat(parts) if parts else torch.zeros((0, screen.REC), device=dev)
+            elif args.scaling == "weak":
                 ctx.run_async(mp, args.seed + rank, None, best_pose, best_score, stream)
                 ids = torch.arange(n_spots, dtype=torch.float32, device=dev)
                 rec = torch.cat([ids[:, None], best_score[:, None], best_pose], 1)
@@ -273,8 +315,8 @@ def main():
     for i in range(args.warmup):
         step(-1 - i)
     torch.cuda.synchronize(dev)
-    ctx.reset_stats()
-    ctx.set_timing(True)
+    work_obj.reset_stats()
+    work_obj.set_timing(True)
     clocks = ClockSampler(local, enabled=(rank == 0 and not args.no_clocks))
     if world > 1:
         dist.barrier()
@@ -290,8 +332,8 @@ def main():
         dist.barrier()
     clk = clocks.stop()
     ms_rank = e0.elapsed_time(e1)
-    st = ctx.stats()
-    ctx.set_timing(False)
+    st = work_obj.stats()
+    work_obj.set_timing(False)
     # whole-job totals and max-over-ranks time
     tot = torch.tensor([st["pairs"], st["poses_scored"], st["kernel_launches"]], dtype=torch.float64, device=cdev)
     tmax = torch.tensor([ms_rank], dtype=torch.float64, device=cdev)
@@ -326,31 +368,37 @@ def main():
     if not args.no_e2e:
         import torch as _t
         pin = lambda a: _t.from_numpy(np.ascontiguousarray(a)).pin_memory().numpy()
-        host = [pin(x) for x in (prob.rec.xyz, prob.rec.q, prob.rec.type, prob.lig.xyz, prob.lig.q, prob.lig.type,
-                                 prob.spots)]
-        n_e2e = args.e2e_steps if args.e2e_steps is not None else max(1, min(args.steps, 2))
+        ligs = prob.ligands if sweep else [prob.lig]
+        rec_h = [pin(x) for x in (prob.rec.xyz, prob.rec.q, prob.rec.type)]
+        lig_h = [[pin(x) for x in (L.xyz, L.q, L.type)] for L in ligs]
+        spot_h = pin(prob.spots)
+        n_e2e = args.e2e_steps if args.e2e_steps is not None else (1 if sweep else max(1, min(args.steps, 2)))
         e2e_ctx_stats = []
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
         for i in range(n_e2e):
-            with vs.Context(*host, sp=sp, device=local) as c2:
-                c2.run(mp, args.seed + rank, None)
-                e2e_ctx_stats.append(c2.stats())
+            # sweep: this rank's share of the ligands (static round robin), one context per ligand
+            for li in (range(rank, len(ligs), world) if sweep else [0]):
+                with vs.Context(*rec_h, *lig_h[li], spot_h, sp=sp, device=local) as c2:
+                    c2.run(mp, (screen.ligand_seed(args.seed, li) if sweep else args.seed + rank), None)
+                    e2e_ctx_stats.append(c2.stats())
         dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=cdev)
         e2e_pairs = torch.tensor([sum(s["pairs"] for s in e2e_ctx_stats)], dtype=torch.float64, device=cdev)
         if world > 1:
             dist.all_reduce(dt, op=dist.ReduceOp.MAX)
             dist.all_reduce(e2e_pairs, op=dist.ReduceOp.SUM)
-        h2d = sum(a.nbytes for a in host)
-        d2h = n_spots * 8 * 4
+        h2d = sum(a.nbytes for a in rec_h) + spot_h.nbytes + sum(a.nbytes for L in lig_h for a in L)
+        d2h = n_spots * 8 * 4 * len(ligs)
         e2e = {"value": float(e2e_pairs.item()) / float(dt.item()), "unit": "pairs/s", "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "steps": n_e2e,
                "what": "vs_create (receptor/ligand/spot upload + per-spot list build) + vs_run (host spot ids) + "
-                       "best poses/scores to host, wall clock"}
+                       "best poses/scores to host, wall clock" + (", per ligand of the library" if sweep else "")}
 
     # ---- scoring-kernel microbenchmark: one vs_score_poses_device batch of device-resident poses
     micro = None
+    if sweep:                       # the microbenchmark uses the first ligand's context
+        ctx = scr.context(0)
     if not args.no_micro:
         n_micro = args.micro_poses
         spot_h, q_h, t_h = synth.make_poses(n_micro, n_spots, 3.0, seed=7)
@@ -383,6 +431,8 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         lens = ctx.list_lengths()
+        if sweep:
+            prob.lig = prob.ligands[0]
         import oracle
         n_s = max(1, min(n_spots, oracle.get_threads()))
         Gs = 2 if args.config in ("medium", "large", "sweep") else min(G, 5)
@@ -399,11 +449,14 @@ def main():
             "metric": METRIC, "value": value, "unit": "pairs/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": args.config, "preset": f"M{args.preset}", "n_rec": cfg.n_rec, "n_lig": cfg.n_lig,
+            "config": {"workload": args.config, "preset": f"M{args.preset}", "n_rec": cfg.n_rec,
+                       "n_lig": ([len(m.q) for m in prob.ligands] if sweep else cfg.n_lig),
                        "n_spots_per_rank": n_spots, "population": cfg.population, "generations": G,
                        "mode": f"cutoff {cutoff:g} A, per-spot lists" if cutoff > 0 else "all pairs",
                        "l2": "flushed between steps (256 MB write inside the timed region)",
-                       "parallelism": (f"dp{world}: independent runs per rank (seed+rank), best-of gathered"
+                       "parallelism": (f"dp{world}: (ligand, spot-chunk) units, largest ligand first, dynamic queue"
+                                       if sweep else
+                                       f"dp{world}: independent runs per rank (seed+rank), best-of gathered"
                                        if args.scaling == "weak" else
                                        f"dp{world}: spots dealt by a dynamic chunk queue, one gather")},
             "poses_per_s": poses / (ms * 1e-3),
@@ -416,7 +469,10 @@ def main():
             "clocks": clk,
         }
         print(json.dumps(line), flush=True)
-    ctx.close()
+    if sweep:
+        scr.close()
+    else:
+        ctx.close()
     if world > 1:
         dist.destroy_process_group()
 

@@ -8,12 +8,12 @@
 namespace vsk {
 
 #ifndef VS_KPAIRS
-#define VS_KPAIRS 4
+#define VS_KPAIRS 3
 #endif
 constexpr int K_PAIRS = VS_KPAIRS;   // slot pairs per thread: one float2 lane-pair per FFMA2
 constexpr int K_SLOTS = 2 * K_PAIRS; // ligand atoms per thread (register blocking)
 #ifndef VS_GPC
-#define VS_GPC 8
+#define VS_GPC 1
 #endif
 constexpr int GROUPS_PER_CTA = VS_GPC;  // warps (ligand-atom groups) per CTA at most
 constexpr int POSES_PER_CTA = 32;   // one pose per lane

@@ -24,7 +24,7 @@
 #include "vs_kernels.cuh"
 
 #ifndef VS_UNROLL
-#define VS_UNROLL 2
+#define VS_UNROLL 4
 #endif
 #ifndef VS_MINB
 #define VS_MINB (16 / GROUPS_PER_CTA)

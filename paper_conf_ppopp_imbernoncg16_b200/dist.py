@@ -66,7 +66,7 @@ def pack(spot_ids: np.ndarray, pose: np.ndarray, score: np.ndarray) -> np.ndarra
 
 
 def gather_records(rec: torch.Tensor, device: torch.device) -> torch.Tensor | None:
-    """Gather variable-length [n, REC] float32 records to rank 0 (one all-gather of counts,
+    """Gather variable-length [n, width] float32 records to rank 0 (one all-gather of counts,
     one gather of padded records).  Returns the concatenation on rank 0, None elsewhere."""
     world = dist.get_world_size()
     rank = dist.get_rank()
@@ -75,7 +75,7 @@ def gather_records(rec: torch.Tensor, device: torch.device) -> torch.Tensor | No
     dist.all_gather(counts, n)
     counts = [int(c.item()) for c in counts]
     mx = max(max(counts), 1)
-    pad = torch.full((mx, REC), float("nan"), dtype=torch.float32, device=device)
+    pad = torch.full((mx, rec.shape[1]), float("nan"), dtype=torch.float32, device=device)
     pad[: rec.shape[0]] = rec.to(device)
     bufs = [torch.empty_like(pad) for _ in range(world)] if rank == 0 else None
     dist.gather(pad, bufs, dst=0)
@@ -94,3 +94,40 @@ def best_per_spot(records: np.ndarray, n_spots: int) -> tuple[np.ndarray, np.nda
             score[s] = r[1]
             pose[s] = r[2:]
     return pose, score
+
+
+# ---------------------------------------------------------------- heterogeneity-aware static split
+def percent_from_times(times: Sequence[float]) -> list[float]:
+    """Eq. (1): Percent = Ex.time(actual GPU) / Ex.time(slowest GPU)."""
+    slowest = max(times)
+    return [t / slowest for t in times]
+
+
+def shares_from_percent(percent: Sequence[float], n_items: int) -> list[tuple[int, int]]:
+    """Each rank's contiguous item range, sized proportional to its speed 1/Percent ("each
+    OpenMP thread then calculates the number of conformations it is in charge of"; reading R27:
+    share proportional to 1/Percent).  Largest-remainder rounding; ranges cover 0..n_items once."""
+    speed = [1.0 / max(p, 1e-12) for p in percent]
+    tot = sum(speed)
+    raw = [n_items * s / tot for s in speed]
+    cnt = [int(math.floor(x)) for x in raw]
+    rem = n_items - sum(cnt)
+    for i in sorted(range(len(raw)), key=lambda i: raw[i] - cnt[i], reverse=True)[:rem]:
+        cnt[i] += 1
+    out, a = [], 0
+    for c in cnt:
+        out.append((a, a + c))
+        a += c
+    return out
+
+
+def warmup_split(warmup: Callable[[], float], n_items: int, device: torch.device) -> tuple[int, int]:
+    """Warm-up phase of PAPER.md §3.3: every rank times a few metaheuristic iterations
+    (``warmup`` returns seconds), the times are max-reduced (here all-gathered: one collective), and
+    each rank takes a share of the items proportional to its speed.  Returns this rank's range."""
+    world, rank = dist.get_world_size(), dist.get_rank()
+    t = torch.tensor([float(warmup())], dtype=torch.float64, device=device)
+    ts = [torch.zeros_like(t) for _ in range(world)]
+    dist.all_gather(ts, t)
+    times = [float(x.item()) for x in ts]
+    return shares_from_percent(percent_from_times(times), n_items)[rank]

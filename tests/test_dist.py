@@ -92,3 +92,33 @@ def test_queue_and_gather_gloo(tmp_path, mode, oracle_mod):
         runs = [o.run(mp_, 42 + r)[1].astype(np.float32) for r in range(2)]
         _, got_sc = vdist.best_per_spot(rec, n)
         np.testing.assert_array_equal(got_sc, np.minimum(runs[0], runs[1]))
+
+
+def test_percent_and_shares():
+    """Eq. (1): Percent = t / t_slowest; shares proportional to 1/Percent (R27)."""
+    p = vdist.percent_from_times([2.0, 1.0, 4.0])
+    assert p == [0.5, 0.25, 1.0]
+    sh = vdist.shares_from_percent(p, 700)
+    sizes = [b - a for a, b in sh]
+    assert sum(sizes) == 700 and sh[0][0] == 0 and sh[-1][1] == 700
+    assert sizes == [200, 400, 100]
+    assert vdist.shares_from_percent([1.0, 1.0], 5) in ([(0, 3), (3, 5)], [(0, 2), (2, 5)])
+
+
+def _warm_worker(rank, world, port, out_path):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    # rank 1 is "two times faster" (P:144: Percent = 0.5)
+    rng = vdist.warmup_split(lambda: 2.0 if rank == 0 else 1.0, 90, torch.device("cpu"))
+    out = [None] * world
+    dist.all_gather_object(out, rng)
+    if rank == 0:
+        np.save(out_path, np.array(out))
+    dist.destroy_process_group()
+
+
+def test_warmup_split_gloo(tmp_path):
+    out = str(tmp_path / "split.npy")
+    mp.spawn(_warm_worker, args=(2, _free_port(), out), nprocs=2, join=True)
+    split = np.load(out)
+    assert split.tolist() == [[0, 30], [30, 90]]
