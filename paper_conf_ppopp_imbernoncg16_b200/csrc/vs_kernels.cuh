@@ -17,8 +17,14 @@ constexpr int K_SLOTS = 2 * K_PAIRS; // ligand atoms per thread (register blocki
 #endif
 constexpr int GROUPS_PER_CTA = VS_GPC;  // warps (ligand-atom groups) per CTA at most
 constexpr int POSES_PER_CTA = 32;   // one pose per lane
-constexpr int TILE = 128;           // receptor atoms per shared-memory stage (4 KB)
-constexpr int NSTAGE = 4;           // bulk-copy ring depth
+#ifndef VS_TILE
+#define VS_TILE 128
+#endif
+#ifndef VS_NSTAGE
+#define VS_NSTAGE 4
+#endif
+constexpr int TILE = VS_TILE;       // receptor atoms per shared-memory stage (32 B each)
+constexpr int NSTAGE = VS_NSTAGE;   // bulk-copy ring depth
 
 enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
 

@@ -90,6 +90,21 @@ def test_score_parity_sampled_full_size(gpu, oracle_mod, name):
     assert np.all(np.isfinite(got))
 
 
+@pytest.mark.parametrize("name,dielectric", [("medium", 0), ("large", 0), ("medium", 1), ("large", 1)])
+def test_all_pairs_full_size_sampled(gpu, oracle_mod, name, dielectric):
+    """Paper mode (no cutoff, every receptor atom) at full size: the fp32 sums over 10k / 30k atoms stay within
+    the 1e-4 tolerance, for the distance-dependent and the constant dielectric (N3)."""
+    prob = synth.make_problem(name)
+    kw = dict(dielectric=1, eps_r=4.0) if dielectric else {}
+    g, o = both(oracle_mod, prob, 0.0, **kw)
+    n = 4096
+    spot, q, t = synth.make_poses(n, prob.cfg.n_spots, 3.0, seed=31)
+    got = g.score_poses(spot, q, t)
+    idx = np.random.default_rng(2).choice(n, 8, replace=False)
+    worst = assert_scores(got[idx], o.score(spot[idx], q[idx], t[idx]), f"{name} all-pairs diel={dielectric}")
+    print(f"worst err/tol {worst:.3f}")
+
+
 @pytest.mark.parametrize("n_lig", [1, 7, 9, 64, 65, 100, 256])
 def test_ragged_ligand_sizes(gpu, oracle_mod, n_lig):
     """Ligands that are not a multiple of the 8-atom register block, and > 64 atoms (chunked CTAs)."""
