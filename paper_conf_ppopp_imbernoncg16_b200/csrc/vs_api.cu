@@ -154,6 +154,7 @@ ScoreArgs base_args(vs_ctx* c) {
   a.n_groups = c->n_groups;
   a.hb_base = c->hb_base;
   a.hb_extra = c->hb_extra;
+  a.hb_max = c->hb_base + (c->hb_extra > 0 ? 1 : 0);
   a.n_chunks = c->n_chunks;
   a.n_lig = c->n_lig;
   a.r2min = c->r2min;
@@ -185,7 +186,7 @@ vs_status score_launch(vs_ctx* c, const ScoreArgs& a, int mode, int n_blocks, cu
   c->launches++;
   c->score_launches++;
   if (a.n_chunks > 1) {
-    CK(launch_finalize(a, mode, n_blocks, st), "finalize kernel launch");
+    CK(launch_finalize(a, mode, a.uniform ? a.nseg * a.fbps : n_blocks, st), "finalize kernel launch");
     c->launches++;
   }
   if (c->timing) CK(cudaEventRecord(e1, st), "cudaEventRecord");
@@ -355,14 +356,12 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     pl.nseg = q.ns;
     pl.seg_spot = q.seg;
     pl.uniform = 1;
-    pl.seg_size = P;
-    pl.bps = (P + POSES_PER_CTA - 1) / POSES_PER_CTA;
     pl.seg_stride = P;
     pl.P = P;
     pl.partial = part ? part + (size_t)k0 * P * c->n_chunks : nullptr;
     q.ls = pl;
-    q.ls.seg_size = m;
-    q.ls.bps = (m + POSES_PER_CTA - 1) / POSES_PER_CTA;
+    plan_uniform(pl, P);
+    plan_uniform(q.ls, m);
     q.ls.J = q.J;
     q.ls.m = m;
     q.ls.seed = seed;

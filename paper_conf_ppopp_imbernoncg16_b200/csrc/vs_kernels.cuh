@@ -39,6 +39,8 @@ struct ScoreArgs {
   const LigSlot* lig;
   int n_groups;              // ligand groups of K_SLOTS slots
   int hb_base, hb_extra;     // group g holds hb_base + (g < hb_extra) H-bond slot pairs, at its end
+  int hb_max;                // max over groups
+  int mixed;                 // 1: lanes map to (pose, group) items of a segment (1-warp CTAs, grid.y = 1)
   int n_chunks;              // ceil(n_groups / GROUPS_PER_CTA)
   int n_lig;                 // real ligand atoms (pair accounting)
   float r2min, rc2, inv_rc2; // rc2 = +inf in all-pairs mode
@@ -47,7 +49,8 @@ struct ScoreArgs {
   int nseg;
   const int* seg_spot;       // [nseg] global spot id
   int uniform;               // 1: every segment has seg_size poses
-  int seg_size, bps;         // uniform
+  int seg_size, bps;         // uniform: poses per segment, scoring blocks per segment
+  int fbps;                  // uniform: 32-pose blocks per segment (finalize)
   const int* blk_prefix;     // non-uniform: [nseg+1]
   const int* pose_prefix;    // non-uniform: [nseg+1]
   // PLAIN
@@ -68,6 +71,9 @@ struct ScoreArgs {
 // launchers (return cudaError_t of the launch)
 cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectric, int n_blocks, cudaStream_t st);
 cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st);
+// lane mapping for a uniform launch of nseg segments of seg_size poses: sets mixed / bps / fbps;
+// returns the number of scoring blocks
+int plan_uniform(ScoreArgs& a, int seg_size);
 cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, uint64_t seed, float T, cudaStream_t st);
 cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, uint64_t seed, int g,
                            float p_mut, float mut_trans, float mut_rot, float T, cudaStream_t st);

@@ -201,13 +201,25 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
   int k, blk;
   locate(a, blockIdx.x, k, blk);
   const int seg_n = a.uniform ? a.seg_size : (__ldg(a.pose_prefix + k + 1) - __ldg(a.pose_prefix + k));
-  const int p0 = blk * POSES_PER_CTA;
-  const int cnt = min(POSES_PER_CTA, seg_n - p0);
   const int spot = __ldg(a.seg_spot + k);
+  int cnt, p, group;
+  if (a.mixed) {
+    // lane -> (pose, ligand group) item of the segment, group-major: fills the lanes when the
+    // segment has few poses (Improve's m = round(f P) poses per spot)
+    const int n_items = seg_n * a.n_groups;
+    const int it0 = blk * POSES_PER_CTA;
+    cnt = min(POSES_PER_CTA, n_items - it0);
+    const int itl = it0 + (lane < cnt ? lane : 0);
+    group = itl / seg_n;
+    p = itl - group * seg_n;
+  } else {
+    const int p0 = blk * POSES_PER_CTA;
+    cnt = min(POSES_PER_CTA, seg_n - p0);
+    p = p0 + (lane < cnt ? lane : 0);
+    group = chunk * GROUPS_PER_CTA + warp;
+  }
   const bool active = lane < cnt;
-  const int p = p0 + (active ? lane : 0);
   const int item = (a.uniform ? k * a.seg_size : __ldg(a.pose_prefix + k)) + p;
-  const int group = chunk * GROUPS_PER_CTA + warp;
 
   // ---- pose of this lane (PLAIN: given; LS: proposal around X[j], R16)
   float4 q, t;
@@ -264,8 +276,9 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
       bulk_g2s(tile[s], src + (size_t)s * TILE, bytes, &full[s]);
     }
   }
-  // warp-uniform number of H-bond pairs in this warp's group (spread evenly over the groups)
-  const int h = a.hb_base + (group < a.hb_extra ? 1 : 0);
+  // warp-uniform number of H-bond pairs in this warp's group (spread evenly over the groups); lanes of
+  // mixed warps hold different groups and all run the largest count (the extra pairs carry zero weight)
+  const int h = a.mixed ? a.hb_max : a.hb_base + (group < a.hb_extra ? 1 : 0);
   double e;
   switch (h) {
 #define VS_CASE(HH) \
@@ -283,7 +296,7 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
     const float score = (float)sum;
     if (active) {
       if (a.n_chunks > 1) {
-        a.partial[(size_t)item * a.n_chunks + chunk] = sum;
+        a.partial[(size_t)item * a.n_chunks + group] = sum;
       } else if (MODE == MODE_PLAIN) {
         const int pidx = a.uniform ? k * a.seg_stride + p : item;
         a.poses[pidx].t.w = score;
@@ -295,9 +308,11 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
         a.poses[jx] = rr;
       }
     }
-    if (lane == 0 && chunk == 0 && a.counters) {
-      atomicAdd(a.counters + 0, (unsigned long long)cnt * (unsigned long long)a.n_lig * (unsigned long long)len);
-      atomicAdd(a.counters + 1, (unsigned long long)cnt);
+    // poses of this CTA counted once: those whose group 0 item it holds
+    const unsigned n0 = __popc(__ballot_sync(0xffffffffu, active && group == 0));
+    if (lane == 0 && n0 && a.counters) {
+      atomicAdd(a.counters + 0, (unsigned long long)n0 * (unsigned long long)a.n_lig * (unsigned long long)len);
+      atomicAdd(a.counters + 1, (unsigned long long)n0);
     }
   }
 }
@@ -309,7 +324,12 @@ __global__ void finalize_kernel(const ScoreArgs a, int n_items_blocks) {
   if (bx >= n_items_blocks) return;
   if (!a.uniform && bx >= __ldg(a.blk_prefix + a.nseg)) return;
   int k, blk;
-  locate(a, bx, k, blk);
+  if (a.uniform) {  // pose blocks (not the scoring launch's lane blocks)
+    k = bx / a.fbps;
+    blk = bx - k * a.fbps;
+  } else {
+    locate(a, bx, k, blk);
+  }
   const int seg_n = a.uniform ? a.seg_size : (__ldg(a.pose_prefix + k + 1) - __ldg(a.pose_prefix + k));
   const int p = blk * POSES_PER_CTA + threadIdx.x;
   if (p >= seg_n) return;
@@ -348,8 +368,8 @@ static cudaError_t launch_diel(const ScoreArgs& a, int diel, dim3 grid, dim3 blo
 
 cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectric, int n_blocks, cudaStream_t st) {
   if (n_blocks <= 0) return cudaSuccess;
-  const int warps = a.n_chunks > 1 ? GROUPS_PER_CTA : a.n_groups;
-  dim3 grid(n_blocks, a.n_chunks), block(warps * 32);
+  const int warps = a.mixed ? 1 : (a.n_chunks > 1 ? GROUPS_PER_CTA : a.n_groups);
+  dim3 grid(n_blocks, a.mixed ? 1 : a.n_chunks), block(warps * 32);
   if (mode == MODE_PLAIN)
     return cutoff ? launch_diel<MODE_PLAIN, true>(a, dielectric, grid, block, st)
                   : launch_diel<MODE_PLAIN, false>(a, dielectric, grid, block, st);
@@ -364,6 +384,23 @@ cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStre
   else
     finalize_kernel<MODE_LS><<<n_blocks, POSES_PER_CTA, 0, st>>>(a, n_blocks);
   return cudaGetLastError();
+}
+
+}  // namespace vsk
+
+namespace vsk {
+
+// Lanes = poses (warp-uniform ligand group, H-bond-specialised loop) unless the segment is short
+// enough that (pose, group) items fill clearly more lanes (e.g. Improve's m = 51 or 13 poses).
+int plan_uniform(ScoreArgs& a, int seg_size) {
+  a.seg_size = seg_size;
+  a.fbps = (seg_size + POSES_PER_CTA - 1) / POSES_PER_CTA;
+  const long lanes_pose = (long)a.fbps * POSES_PER_CTA * a.n_groups;
+  const long items = (long)seg_size * a.n_groups;
+  const long lanes_mixed = (items + POSES_PER_CTA - 1) / POSES_PER_CTA * POSES_PER_CTA;
+  a.mixed = (GROUPS_PER_CTA == 1 && a.n_groups > 1 && lanes_mixed * 100 < lanes_pose * 95) ? 1 : 0;
+  a.bps = a.mixed ? (int)(lanes_mixed / POSES_PER_CTA) : a.fbps;
+  return a.bps;
 }
 
 }  // namespace vsk
