@@ -8,6 +8,7 @@
 // end (best pose + score per spot).
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -92,6 +93,7 @@ struct vs_ctx {
   LigSlot* d_lig = nullptr;
   int* d_iota = nullptr;
   unsigned long long* d_counters = nullptr;
+  uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
   cudaStream_t stream = nullptr;
   cudaStream_t sub[NSUB] = {};          // per-spot-group streams of vs_run
   cudaEvent_t ev_fork = nullptr, ev_join[NSUB] = {};
@@ -104,6 +106,11 @@ struct vs_ctx {
   size_t ev_used = 0;
   double score_ms_acc = 0.0;
   uint64_t timed_acc = 0;
+  // CUDA graph of vs_run (captured on the second identical call)
+  bool graphs = true, capturing = false, has_last = false;
+  cudaGraphExec_t gexec = nullptr;
+  unsigned char gkey[160] = {}, last_key[160] = {};
+  uint64_t g_launches = 0, g_score_launches = 0;
 };
 
 namespace {
@@ -164,12 +171,14 @@ ScoreArgs base_args(vs_ctx* c) {
   a.hbD = c->hbD;
   a.T = c->T;
   a.counters = c->d_counters;
+  a.seedp = c->d_seed;
   return a;
 }
 
 vs_status score_launch(vs_ctx* c, const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st) {
   cudaEvent_t e0 = nullptr, e1 = nullptr;
-  if (c->timing) {
+  const bool timed = c->timing && !c->capturing;  // graph replays are timed by the caller as a whole
+  if (timed) {
     if (c->ev_used + 2 > c->ev.size()) {
       for (int i = 0; i < 64; ++i) {
         cudaEvent_t e;
@@ -189,7 +198,7 @@ vs_status score_launch(vs_ctx* c, const ScoreArgs& a, int mode, int n_blocks, cu
     CK(launch_finalize(a, mode, a.uniform ? a.nseg * a.fbps : n_blocks, st), "finalize kernel launch");
     c->launches++;
   }
-  if (c->timing) CK(cudaEventRecord(e1, st), "cudaEventRecord");
+  if (timed) CK(cudaEventRecord(e1, st), "cudaEventRecord");
   return VS_OK;
 }
 
@@ -231,6 +240,19 @@ vs_status trace_idx(vs_ctx* c, Tracer* tr, cudaStream_t st, int stage, int g, in
   return VS_OK;
 }
 
+// Everything one run's enqueued work depends on except the seed (also the CUDA-graph cache key).
+struct Body {
+  vs_mh_params mp;
+  int m, ns;
+  int* seg;
+  PoseRec *SA, *SB, *CC;
+  int* JJ;
+  double* part;
+  float *best_pose, *best_score;
+};
+
+static_assert(sizeof(Body) <= 160, "graph key storage");
+
 // One group of spots running Algorithm 1 on its own stream.
 struct Group {
   int ns = 0;
@@ -263,9 +285,9 @@ vs_status improve_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, PoseR
 }
 
 // Initialize(S): random population, scored, improved when f > 0, sorted.
-vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, uint64_t seed, int m, Tracer* tr) {
+vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, Tracer* tr) {
   const int P = mp->population;
-  CK(launch_init(q.S, q.ns, P, q.seg, seed, c->T, q.st), "init launch");
+  CK(launch_init(q.S, q.ns, P, q.seg, c->d_seed, c->T, q.st), "init launch");
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_INIT, 0, 0, q.ns, P, q.S);
   if (r != VS_OK) return r;
@@ -282,9 +304,9 @@ vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, uint64_t s
 }
 
 // One pass of the while-loop body: Select + Combine, score, Improve, Include.
-vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, uint64_t seed, int m, int g, Tracer* tr) {
+vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, int g, Tracer* tr) {
   const int P = mp->population;
-  CK(launch_combine(q.S, q.C, q.ns, P, q.seg, seed, g, mp->p_mut, mp->mut_trans, mp->mut_rot, c->T, q.st),
+  CK(launch_combine(q.S, q.C, q.ns, P, q.seg, c->d_seed, g, mp->p_mut, mp->mut_trans, mp->mut_rot, c->T, q.st),
      "combine launch");
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_COMBINED, g, 0, q.ns, P, q.C);
@@ -299,6 +321,61 @@ vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, uint64_t seed, i
   std::swap(q.S, q.S2);
   q.in_b = !q.in_b;
   return trace_poses(c, tr, q.st, VS_TRACE_INCLUDED, g, 0, q.ns, P, q.S);
+}
+
+// Everything a run enqueues after its inputs are on the device (the part a CUDA graph captures).
+vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
+  const vs_mh_params* mp = &b.mp;
+  const int P = mp->population, m = b.m, ns = b.ns;
+  // Spots are independent (P:84): split them into groups whose generation loops run on separate
+  // streams, enqueued generation by generation, so one group's kernels fill the wave tails of
+  // another's.
+  const int G = tr ? 1 : std::max(1, std::min(NSUB, ns / 64));
+  Group grp[NSUB];
+  CK(cudaEventRecord(c->ev_fork, st), "event record");
+  for (int gi = 0; gi < G; ++gi) {
+    const int k0 = (int)((int64_t)ns * gi / G), k1 = (int)((int64_t)ns * (gi + 1) / G);
+    Group& q = grp[gi];
+    q.ns = k1 - k0;
+    q.seg = b.seg + k0;
+    q.S = b.SA + (size_t)k0 * P;
+    q.S2 = b.SB + (size_t)k0 * P;
+    q.C = b.CC + (size_t)k0 * P;
+    q.J = b.JJ + (size_t)k0 * m;
+    q.st = G > 1 ? c->sub[gi] : st;
+    if (G > 1) CK(cudaStreamWaitEvent(q.st, c->ev_fork, 0), "stream wait");
+    ScoreArgs& pl = q.plain;
+    pl = base_args(c);
+    pl.nseg = q.ns;
+    pl.seg_spot = q.seg;
+    pl.uniform = 1;
+    pl.seg_stride = P;
+    pl.P = P;
+    pl.partial = b.part ? b.part + (size_t)k0 * P * c->n_chunks : nullptr;
+    q.ls = pl;
+    plan_uniform(pl, P);
+    plan_uniform(q.ls, m);
+    q.ls.J = q.J;
+    q.ls.m = m;
+    q.ls.ls_trans = mp->ls_trans;
+    q.ls.ls_rot = mp->ls_rot;
+    q.plain_blocks = q.ns * pl.bps;
+    q.ls_blocks = q.ns * q.ls.bps;
+  }
+  vs_status r;
+  for (int gi = 0; gi < G; ++gi)
+    if ((r = gen_initialize(c, grp[gi], mp, m, tr)) != VS_OK) return r;
+  for (int g = 1; g <= mp->generations; ++g)         // End(S): fixed G (R20)
+    for (int gi = 0; gi < G; ++gi)
+      if ((r = gen_step(c, grp[gi], mp, m, g, tr)) != VS_OK) return r;
+  if (G > 1)
+    for (int gi = 0; gi < G; ++gi) {
+      CK(cudaEventRecord(c->ev_join[gi], grp[gi].st), "event record");
+      CK(cudaStreamWaitEvent(st, c->ev_join[gi], 0), "stream wait");
+    }
+  CK(launch_best(grp[0].in_b ? b.SB : b.SA, ns, P, b.best_pose, b.best_score, st), "best launch");
+  c->launches++;
+  return VS_OK;
 }
 
 // The generation loop (Algorithm 1) for n_sel spots, all on stream st.
@@ -328,61 +405,59 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     CK(cudaMemcpyAsync(seg, spot_ids, sizeof(int) * ns, cudaMemcpyHostToDevice, st), "H2D spot ids");
   else
     CK(cudaMemcpyAsync(seg, c->d_iota, sizeof(int) * ns, cudaMemcpyDeviceToDevice, st), "D2D spot ids");
-  PoseRec* SA = (PoseRec*)c->buf[B_SA].p;
-  PoseRec* SB = (PoseRec*)c->buf[B_SB].p;
-  PoseRec* CC = (PoseRec*)c->buf[B_C].p;
-  int* JJ = (int*)c->buf[B_J].p;
-  double* part = (double*)c->buf[B_PART].p;
+  // the seed lives in device memory so that a captured graph can be replayed for any seed
+  CK(cudaMemcpyAsync(c->d_seed, &seed, sizeof(uint64_t), cudaMemcpyHostToDevice, st), "H2D seed");
+  Body b;
+  std::memset(&b, 0, sizeof(b));  // padding bytes take part in the graph-cache key comparison
+  b.mp = *mp;
+  b.m = m;
+  b.ns = ns;
+  b.seg = seg;
+  b.SA = (PoseRec*)c->buf[B_SA].p;
+  b.SB = (PoseRec*)c->buf[B_SB].p;
+  b.CC = (PoseRec*)c->buf[B_C].p;
+  b.JJ = (int*)c->buf[B_J].p;
+  b.part = (double*)c->buf[B_PART].p;
+  b.best_pose = d_best_pose;
+  b.best_score = d_best_score;
+  if (tr || !c->graphs) return enqueue_body(c, b, st, tr);
 
-  // Spots are independent (P:84): split them into groups whose generation loops run on separate
-  // streams, enqueued generation by generation, so one group's kernels fill the wave tails of
-  // another's.
-  const int G = tr ? 1 : std::max(1, std::min(NSUB, ns / 64));
-  Group grp[NSUB];
-  CK(cudaEventRecord(c->ev_fork, st), "event record");
-  for (int gi = 0; gi < G; ++gi) {
-    const int k0 = (int)((int64_t)ns * gi / G), k1 = (int)((int64_t)ns * (gi + 1) / G);
-    Group& q = grp[gi];
-    q.ns = k1 - k0;
-    q.seg = seg + k0;
-    q.S = SA + (size_t)k0 * P;
-    q.S2 = SB + (size_t)k0 * P;
-    q.C = CC + (size_t)k0 * P;
-    q.J = JJ + (size_t)k0 * m;
-    q.st = G > 1 ? c->sub[gi] : st;
-    if (G > 1) CK(cudaStreamWaitEvent(q.st, c->ev_fork, 0), "stream wait");
-    ScoreArgs& pl = q.plain;
-    pl = base_args(c);
-    pl.nseg = q.ns;
-    pl.seg_spot = q.seg;
-    pl.uniform = 1;
-    pl.seg_stride = P;
-    pl.P = P;
-    pl.partial = part ? part + (size_t)k0 * P * c->n_chunks : nullptr;
-    q.ls = pl;
-    plan_uniform(pl, P);
-    plan_uniform(q.ls, m);
-    q.ls.J = q.J;
-    q.ls.m = m;
-    q.ls.seed = seed;
-    q.ls.ls_trans = mp->ls_trans;
-    q.ls.ls_rot = mp->ls_rot;
-    q.plain_blocks = q.ns * pl.bps;
-    q.ls_blocks = q.ns * q.ls.bps;
+  // CUDA graph of the whole run: captured on the second identical call, replayed afterwards
+  // (the ~4 + 2 L launches per generation and spot group then cost one graph launch).
+  const bool same_as_cached = c->gexec && std::memcmp(&b, &c->gkey, sizeof(Body)) == 0;
+  if (same_as_cached) {
+    CK(cudaGraphLaunch(c->gexec, st), "graph launch");
+    c->launches += c->g_launches;
+    c->score_launches += c->g_score_launches;
+    return VS_OK;
   }
-  vs_status r;
-  for (int gi = 0; gi < G; ++gi)
-    if ((r = gen_initialize(c, grp[gi], mp, seed, m, tr)) != VS_OK) return r;
-  for (int g = 1; g <= mp->generations; ++g)         // End(S): fixed G (R20)
-    for (int gi = 0; gi < G; ++gi)
-      if ((r = gen_step(c, grp[gi], mp, seed, m, g, tr)) != VS_OK) return r;
-  if (G > 1)
-    for (int gi = 0; gi < G; ++gi) {
-      CK(cudaEventRecord(c->ev_join[gi], grp[gi].st), "event record");
-      CK(cudaStreamWaitEvent(st, c->ev_join[gi], 0), "stream wait");
-    }
-  CK(launch_best(grp[0].in_b ? SB : SA, ns, P, d_best_pose, d_best_score, st), "best launch");
-  c->launches++;
+  const bool seen = c->has_last && std::memcmp(&b, &c->last_key, sizeof(Body)) == 0;
+  std::memcpy(&c->last_key, &b, sizeof(Body));
+  c->has_last = true;
+  if (!seen) return enqueue_body(c, b, st, tr);
+  if (c->gexec) {
+    cudaGraphExecDestroy(c->gexec);
+    c->gexec = nullptr;
+  }
+  const uint64_t l0 = c->launches, s0 = c->score_launches;
+  CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal), "begin capture");
+  c->capturing = true;
+  vs_status r = enqueue_body(c, b, st, tr);
+  c->capturing = false;
+  cudaGraph_t graph = nullptr;
+  cudaError_t e = cudaStreamEndCapture(st, &graph);
+  if (r != VS_OK) {
+    if (graph) cudaGraphDestroy(graph);
+    return r;
+  }
+  CK(e, "end capture");
+  e = cudaGraphInstantiate(&c->gexec, graph, 0);
+  cudaGraphDestroy(graph);
+  CK(e, "graph instantiate");
+  std::memcpy(&c->gkey, &b, sizeof(Body));
+  c->g_launches = c->launches - l0;
+  c->g_score_launches = c->score_launches - s0;
+  CK(cudaGraphLaunch(c->gexec, st), "graph launch");
   return VS_OK;
 }
 
@@ -679,6 +754,11 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   CKT(cudaMalloc(&c->d_iota, sizeof(int) * n_spots), "alloc");
   CKT(cudaMemcpy(c->d_iota, iota.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
   CKT(cudaMalloc(&c->d_counters, sizeof(unsigned long long) * 2), "alloc");
+  CKT(cudaMalloc(&c->d_seed, sizeof(uint64_t)), "alloc");
+  {
+    const char* gv = std::getenv("VS_GRAPHS");
+    c->graphs = !(gv && gv[0] == '0');
+  }
   CKT(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 2), "memset");
   CKT(cudaStreamSynchronize(c->stream), "sync");
   free_tmp();
@@ -781,7 +861,9 @@ void vs_destroy(vs_ctx* c) {
   cudaDeviceSynchronize();
   for (auto& b : c->buf) b.release();
   for (auto e : c->ev) cudaEventDestroy(e);
-  void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_lig, c->d_iota, c->d_counters};
+  if (c->gexec) cudaGraphExecDestroy(c->gexec);
+  void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_lig, c->d_iota, c->d_counters,
+                  c->d_seed};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (c->stream) cudaStreamDestroy(c->stream);

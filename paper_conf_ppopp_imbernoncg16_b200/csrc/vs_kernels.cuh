@@ -62,7 +62,7 @@ struct ScoreArgs {
   // LS (Improve step): X[k*P + J[k*m + jj]] perturbed, scored, accepted if better
   const int* J;
   int m, P;
-  uint64_t seed;
+  const uint64_t* seedp;      // run seed in device memory (graph replays need no new parameters)
   int g, l;
   float ls_trans, ls_rot, T;
   unsigned long long* counters;  // [0] pairs, [1] poses
@@ -74,8 +74,8 @@ cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStre
 // lane mapping for a uniform launch of nseg segments of seg_size poses: sets mixed / bps / fbps;
 // returns the number of scoring blocks
 int plan_uniform(ScoreArgs& a, int seg_size);
-cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, uint64_t seed, float T, cudaStream_t st);
-cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, uint64_t seed, int g,
+cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, cudaStream_t st);
+cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, int g,
                            float p_mut, float mut_trans, float mut_rot, float T, cudaStream_t st);
 // sort (score, index) per segment: mode 0: select best m indices -> J;
 // mode 1: sort S -> S_out; mode 2: include: best P of S ++ C -> S_out

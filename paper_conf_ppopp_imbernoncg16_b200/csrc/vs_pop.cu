@@ -12,7 +12,8 @@
 
 namespace vsk {
 
-__global__ void init_kernel(PoseRec* S, int n_sel, int P, const int* seg_spot, uint64_t seed, float T) {
+__global__ void init_kernel(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T) {
+  const uint64_t seed = *seedp;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= n_sel * P) return;
   const int k = idx / P, i = idx - k * P;
@@ -26,8 +27,9 @@ __global__ void init_kernel(PoseRec* S, int n_sel, int P, const int* seg_spot, u
 
 // child j of generation g from the sorted population S (rank = index)
 __global__ void combine_kernel(const PoseRec* __restrict__ S, PoseRec* __restrict__ C, int n_sel, int P,
-                               const int* seg_spot, uint64_t seed, int g, float p_mut, float mut_trans, float mut_rot,
-                               float T) {
+                               const int* seg_spot, const uint64_t* seedp, int g, float p_mut, float mut_trans,
+                               float mut_rot, float T) {
+  const uint64_t seed = *seedp;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= n_sel * P) return;
   const int k = idx / P, j = idx - k * P;
@@ -242,14 +244,14 @@ __global__ void scatter_kernel(int64_t n, const int32_t* spot, const float* q, c
 // ---------------------------------------------------------------- launchers
 static inline int nblk(int64_t n, int b) { return (int)((n + b - 1) / b); }
 
-cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, uint64_t seed, float T, cudaStream_t st) {
-  init_kernel<<<nblk((int64_t)n_sel * P, 128), 128, 0, st>>>(S, n_sel, P, seg_spot, seed, T);
+cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, cudaStream_t st) {
+  init_kernel<<<nblk((int64_t)n_sel * P, 128), 128, 0, st>>>(S, n_sel, P, seg_spot, seedp, T);
   return cudaGetLastError();
 }
 
-cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, uint64_t seed, int g,
+cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, int g,
                            float p_mut, float mut_trans, float mut_rot, float T, cudaStream_t st) {
-  combine_kernel<<<nblk((int64_t)n_sel * P, 128), 128, 0, st>>>(S, C, n_sel, P, seg_spot, seed, g, p_mut, mut_trans,
+  combine_kernel<<<nblk((int64_t)n_sel * P, 128), 128, 0, st>>>(S, C, n_sel, P, seg_spot, seedp, g, p_mut, mut_trans,
                                                                 mut_rot, T);
   return cudaGetLastError();
 }

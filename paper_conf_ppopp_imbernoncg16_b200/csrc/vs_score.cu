@@ -237,7 +237,7 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
     q = r.q;
     t = r.t;
     old_score = r.t.w;
-    perturb(q, t, a.ls_trans, a.ls_rot, a.T, a.seed, (uint32_t)j, (uint32_t)spot, (uint32_t)a.g, TAG_LS,
+    perturb(q, t, a.ls_trans, a.ls_rot, a.T, *a.seedp, (uint32_t)j, (uint32_t)spot, (uint32_t)a.g, TAG_LS,
             2u * (uint32_t)a.l);
   }
 
@@ -348,7 +348,7 @@ __global__ void finalize_kernel(const ScoreArgs a, int n_items_blocks) {
     PoseRec r = a.poses[jx];
     if (score < r.t.w) {
       float4 q = r.q, t = r.t;
-      perturb(q, t, a.ls_trans, a.ls_rot, a.T, a.seed, (uint32_t)j, (uint32_t)spot, (uint32_t)a.g, TAG_LS,
+      perturb(q, t, a.ls_trans, a.ls_rot, a.T, *a.seedp, (uint32_t)j, (uint32_t)spot, (uint32_t)a.g, TAG_LS,
               2u * (uint32_t)a.l);
       r.q = q;
       r.t = make_float4(t.x, t.y, t.z, score);

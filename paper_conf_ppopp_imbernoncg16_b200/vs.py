@@ -174,7 +174,10 @@ class Context:
 
     def close(self):
         if getattr(self, "h", None):
-            load().vs_destroy(self.h)
+            try:
+                load().vs_destroy(self.h)
+            except TypeError:  # interpreter shutdown: module globals already torn down
+                pass
             self.h = None
 
     __del__ = close
