@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--config", default="medium")
     ap.add_argument("--preset", type=int, default=3)
     ap.add_argument("--generations", type=int, default=None, help="override the config's G")
+    ap.add_argument("--ls-neighbours", type=int, default=1, help="K proposals per Improve step (N4)")
     ap.add_argument("--mode", choices=["cutoff", "allpairs"], default="cutoff")
     ap.add_argument("--scaling", choices=["weak", "strong"], default="weak")
     ap.add_argument("--seed", type=int, default=42)
@@ -233,7 +234,7 @@ def main():
     G = cfg.generations if args.generations is None else args.generations
     cutoff = 12.0 if args.mode == "cutoff" else 0.0
     sp = vs.score_params(cutoff=cutoff)
-    mp = vs.mh_preset(args.preset, population=cfg.population, generations=G)
+    mp = vs.mh_preset(args.preset, population=cfg.population, generations=G, ls_neighbours=args.ls_neighbours)
     sweep = cfg.n_ligands > 1
     n_spots = cfg.n_spots
     stream = torch.cuda.Stream(device=dev)

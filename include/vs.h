@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define VS_ABI_VERSION 1
+#define VS_ABI_VERSION 2
 
 #if defined(__GNUC__)
 #define VS_API __attribute__((visibility("default")))
@@ -89,6 +89,8 @@ typedef struct {
 typedef struct {
   int population, generations, ls_steps;
   float improve_frac, p_mut, mut_trans, mut_rot, ls_trans, ls_rot;
+  int ls_neighbours;  /* K in [1, 64] proposals per Improve step scored together, the best replaces the
+                         element if strictly better; 1 = first-improvement hill climbing */
 } vs_mh_params;
 
 VS_API void vs_score_params_default(vs_score_params* out);
@@ -97,7 +99,7 @@ VS_API void vs_score_params_default(vs_score_params* out);
  *   M1 GA: P 64, f 0;  M2: P 64, f 1, L 8;  M3: P 64, f 0.2, L 8;
  *   M4: P 1024, G 0, f 1, L 8 ("only one step").
  *   G = 50 for M1-M3 (the paper does not report it, R22); p_mut 0.1,
- *   mut 1.0 A / 0.25, ls 0.5 A / 0.10.
+ *   mut 1.0 A / 0.25, ls 0.5 A / 0.10, ls_neighbours 1.
  * Returns VS_ERR_INVALID_ARGUMENT for another m or out == NULL. */
 VS_API vs_status vs_mh_preset(int m, vs_mh_params* out);
 

@@ -44,7 +44,8 @@ class ScoreParams(C.Structure):
 class MHParams(C.Structure):
     _fields_ = [("population", C.c_int), ("generations", C.c_int), ("ls_steps", C.c_int),
                 ("improve_frac", C.c_float), ("p_mut", C.c_float), ("mut_trans", C.c_float),
-                ("mut_rot", C.c_float), ("ls_trans", C.c_float), ("ls_rot", C.c_float)]
+                ("mut_rot", C.c_float), ("ls_trans", C.c_float), ("ls_rot", C.c_float),
+                ("ls_neighbours", C.c_int)]
 
 
 _lib = None
@@ -83,6 +84,8 @@ def lib():
                                         f32p, f32p]
         L.vso_ls_proposal.argtypes = [vp, C.POINTER(MHParams), C.c_uint64, C.c_int32, C.c_int32, C.c_int32,
                                       C.c_int32, f32p, f32p]
+        L.vso_ls_proposal_k.argtypes = [vp, C.POINTER(MHParams), C.c_uint64, C.c_int32, C.c_int32, C.c_int32,
+                                        C.c_int32, C.c_int32, f32p, f32p]
         L.vso_improve_count.argtypes = [C.POINTER(MHParams)]
         L.vso_select_improve.argtypes = [f64p, C.c_int32, C.c_int32, i32p]
         L.vso_include.argtypes = [f64p, f64p, C.c_int32, i32p]
@@ -247,8 +250,8 @@ class Oracle:
         lib().vso_combine_child(self.h, C.byref(mp), seed, spot, g, j, _p(S, C.c_float), _p(o, C.c_float))
         return o
 
-    def ls_proposal(self, mp: MHParams, seed: int, spot: int, g: int, l: int, j: int, pose) -> np.ndarray:
+    def ls_proposal(self, mp: MHParams, seed: int, spot: int, g: int, l: int, j: int, pose, k: int = 0) -> np.ndarray:
         p = np.ascontiguousarray(pose, np.float32).reshape(7)
         o = np.zeros(7, np.float32)
-        lib().vso_ls_proposal(self.h, C.byref(mp), seed, spot, g, l, j, _p(p, C.c_float), _p(o, C.c_float))
+        lib().vso_ls_proposal_k(self.h, C.byref(mp), seed, spot, g, l, k, j, _p(p, C.c_float), _p(o, C.c_float))
         return o

@@ -309,19 +309,26 @@ struct MH {
   }
 
   // Improve(Scom): local search in the neighbourhood of the best m
-  // elements (R16, R17): first-improvement hill climbing, L steps, strict <.
+  // elements (R16, R17): L steps, strict <.  With K = ls_neighbours proposals
+  // per step the best of the K replaces the element if it is strictly better
+  // (lowest k on ties; K = 1 is first-improvement hill climbing).
   void improve(std::vector<Pose>& X, int g) const {
     int P = (int)X.size();
     std::vector<double> sc(P);
     for (int i = 0; i < P; ++i) sc[i] = X[i].score;
     std::vector<int> J(m);
     vso_select_improve(sc.data(), P, m, J.data());
+    const int K = mp.ls_neighbours;
     for (int l = 0; l < mp.ls_steps; ++l) {
       for (int j : J) {
-        Pose cand = X[j];
-        perturb(cand, mp.ls_trans, mp.ls_rot, c->T, seed, j, s, g, TAG_LS, 2 * l);
-        cand.score = score_pose(c, s, cand.q, cand.t);
-        if (cand.score < X[j].score) X[j] = cand;
+        Pose best = X[j];
+        for (int k = 0; k < K; ++k) {
+          Pose cand = X[j];
+          perturb(cand, mp.ls_trans, mp.ls_rot, c->T, seed, j, s, g, TAG_LS, 2 * (l * K + k));
+          cand.score = score_pose(c, s, cand.q, cand.t);
+          if (cand.score < best.score) best = cand;
+        }
+        X[j] = best;
       }
     }
   }
@@ -361,6 +368,7 @@ vso_status check_mh(const vso_mh_params* mp) {
   if (mp->generations < 0) return fail(VSO_ERR_INVALID_ARGUMENT, "generations must be >= 0");
   if (mp->generations > 0 && mp->population < 2) return fail(VSO_ERR_INVALID_ARGUMENT, "population must be >= 2 when generations > 0");
   if (mp->ls_steps < 0) return fail(VSO_ERR_INVALID_ARGUMENT, "ls_steps must be >= 0");
+  if (mp->ls_neighbours < 1 || mp->ls_neighbours > 64) return fail(VSO_ERR_INVALID_ARGUMENT, "ls_neighbours must be in [1, 64]");
   if (!(mp->improve_frac >= 0.0f && mp->improve_frac <= 1.0f)) return fail(VSO_ERR_INVALID_ARGUMENT, "improve_frac must be in [0, 1]");
   if (!(mp->p_mut >= 0.0f && mp->p_mut <= 1.0f)) return fail(VSO_ERR_INVALID_ARGUMENT, "p_mut must be in [0, 1]");
   const float st[4] = {mp->mut_trans, mp->mut_rot, mp->ls_trans, mp->ls_rot};
@@ -402,6 +410,7 @@ vso_status vso_mh_preset(int m, vso_mh_params* o) {
   o->mut_rot = 0.25f;
   o->ls_trans = 0.5f;
   o->ls_rot = 0.10f;
+  o->ls_neighbours = 1;
   return VSO_OK;
 }
 
@@ -554,7 +563,7 @@ vso_status vso_run_d(vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t
 
 void vso_destroy(vso_ctx* c) { delete c; }
 const char* vso_last_error(void) { return g_err.c_str(); }
-int vso_abi_version(void) { return 1; }
+int vso_abi_version(void) { return 2; }
 
 void vso_set_threads(int n) {
 #ifdef _OPENMP
@@ -617,9 +626,14 @@ void vso_combine_child(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed,
 
 void vso_ls_proposal(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot, int32_t g,
                      int32_t l, int32_t j, const float in[7], float out[7]) {
+  vso_ls_proposal_k(c, mp, seed, spot, g, l, 0, j, in, out);
+}
+
+void vso_ls_proposal_k(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot, int32_t g,
+                       int32_t l, int32_t k, int32_t j, const float in[7], float out[7]) {
   Pose p;
   to_pose(in, p);
-  perturb(p, mp->ls_trans, mp->ls_rot, c->T, seed, j, spot, g, TAG_LS, 2 * l);
+  perturb(p, mp->ls_trans, mp->ls_rot, c->T, seed, j, spot, g, TAG_LS, 2 * (l * mp->ls_neighbours + k));
   from_pose(p, out);
 }
 

@@ -40,6 +40,7 @@ typedef struct {
 typedef struct {
   int population, generations, ls_steps;
   float improve_frac, p_mut, mut_trans, mut_rot, ls_trans, ls_rot;
+  int ls_neighbours;   /* K proposals per Improve step, best-of-K accepted; 1 = hill climbing */
 } vso_mh_params;
 
 void        vso_score_params_default(vso_score_params* out);
@@ -77,6 +78,9 @@ void vso_combine_child(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed,
                        int32_t g, int32_t j, const float* S_sorted /*[P][7]*/, float pose_out[7]);
 void vso_ls_proposal(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot,
                      int32_t g, int32_t l, int32_t j, const float pose_in[7], float pose_out[7]);
+/* proposal k (0 <= k < ls_neighbours) of Improve step l for individual j */
+void vso_ls_proposal_k(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot,
+                       int32_t g, int32_t l, int32_t k, int32_t j, const float pose_in[7], float pose_out[7]);
 int32_t vso_improve_count(const vso_mh_params* mp);          /* m of Improve */
 /* J = indices of the best m of scores[P] by (score, index) */
 void vso_select_improve(const double* scores, int32_t P, int32_t m, int32_t* J_out);

@@ -67,7 +67,7 @@ struct DevBuf {
 constexpr int NSUB = 4;  // spot groups (streams) of one vs_run
 
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
-           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_COUNT };
+           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_COUNT };
 
 bool finite_arr(const float* p, int64_t n) {
   for (int64_t i = 0; i < n; ++i)
@@ -134,6 +134,8 @@ vs_status check_mh(const vs_mh_params* mp) {
   if (mp->generations > 0 && mp->population < 2)
     return set_err(VS_ERR_INVALID_ARGUMENT, "population must be >= 2 when generations > 0");
   if (mp->ls_steps < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "ls_steps must be >= 0");
+  if (mp->ls_neighbours < 1 || mp->ls_neighbours > 64)
+    return set_err(VS_ERR_INVALID_ARGUMENT, "ls_neighbours must be in [1, 64]");
   if (!(mp->improve_frac >= 0.0f && mp->improve_frac <= 1.0f)) return set_err(VS_ERR_INVALID_ARGUMENT, "improve_frac must be in [0, 1]");
   if (!(mp->p_mut >= 0.0f && mp->p_mut <= 1.0f)) return set_err(VS_ERR_INVALID_ARGUMENT, "p_mut must be in [0, 1]");
   const float st[4] = {mp->mut_trans, mp->mut_rot, mp->ls_trans, mp->ls_rot};
@@ -248,6 +250,7 @@ struct Body {
   PoseRec *SA, *SB, *CC;
   int* JJ;
   double* part;
+  float* pscore;
   float *best_pose, *best_score;
 };
 
@@ -279,6 +282,10 @@ vs_status improve_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, PoseR
     a.g = g;
     a.l = l;
     if ((r = score_launch(c, a, MODE_LS, q.ls_blocks, q.st)) != VS_OK) return r;
+    if (a.K > 1) {
+      CK(launch_lsk_accept(a, q.st), "accept launch");
+      c->launches++;
+    }
     if ((r = trace_poses(c, tr, q.st, VS_TRACE_LS, g, l, q.ns, P, X)) != VS_OK) return r;
   }
   return VS_OK;
@@ -351,12 +358,14 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     pl.uniform = 1;
     pl.seg_stride = P;
     pl.P = P;
-    pl.partial = b.part ? b.part + (size_t)k0 * P * c->n_chunks : nullptr;
+    pl.partial = b.part ? b.part + (size_t)k0 * std::max(P, m * mp->ls_neighbours) * c->n_chunks : nullptr;
     q.ls = pl;
     plan_uniform(pl, P);
-    plan_uniform(q.ls, m);
+    plan_uniform(q.ls, m * mp->ls_neighbours);
     q.ls.J = q.J;
     q.ls.m = m;
+    q.ls.K = mp->ls_neighbours;
+    q.ls.pscore = b.pscore ? b.pscore + (size_t)k0 * m * mp->ls_neighbours : nullptr;
     q.ls.ls_trans = mp->ls_trans;
     q.ls.ls_rot = mp->ls_rot;
     q.plain_blocks = q.ns * pl.bps;
@@ -399,7 +408,9 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   CK(c->buf[B_SB].ensure(pop_bytes), "alloc");
   CK(c->buf[B_C].ensure(pop_bytes), "alloc");
   CK(c->buf[B_J].ensure(sizeof(int) * (size_t)ns * m), "alloc");
-  if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * (size_t)ns * P * c->n_chunks), "alloc");
+  const size_t items = (size_t)ns * std::max(P, m * mp->ls_neighbours);
+  if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * items * c->n_chunks), "alloc");
+  if (mp->ls_neighbours > 1) CK(c->buf[B_PSCORE].ensure(sizeof(float) * (size_t)ns * m * mp->ls_neighbours), "alloc");
   int* seg = (int*)c->buf[B_SEG].p;
   if (spot_ids)
     CK(cudaMemcpyAsync(seg, spot_ids, sizeof(int) * ns, cudaMemcpyHostToDevice, st), "H2D spot ids");
@@ -418,6 +429,7 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   b.CC = (PoseRec*)c->buf[B_C].p;
   b.JJ = (int*)c->buf[B_J].p;
   b.part = (double*)c->buf[B_PART].p;
+  b.pscore = mp->ls_neighbours > 1 ? (float*)c->buf[B_PSCORE].p : nullptr;
   b.best_pose = d_best_pose;
   b.best_score = d_best_score;
   if (tr || !c->graphs) return enqueue_body(c, b, st, tr);
@@ -532,6 +544,7 @@ vs_status vs_mh_preset(int m, vs_mh_params* o) {
   o->mut_rot = 0.25f;
   o->ls_trans = 0.5f;
   o->ls_rot = 0.10f;
+  o->ls_neighbours = 1;
   return VS_OK;
 }
 

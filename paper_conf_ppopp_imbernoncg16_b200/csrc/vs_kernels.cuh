@@ -62,6 +62,8 @@ struct ScoreArgs {
   // LS (Improve step): X[k*P + J[k*m + jj]] perturbed, scored, accepted if better
   const int* J;
   int m, P;
+  int K;                     // proposals per Improve step (segment item p: element p / K, proposal p % K)
+  float* pscore;             // K > 1: proposal scores [nseg][m][K], accepted by lsk_accept_kernel
   const uint64_t* seedp;      // run seed in device memory (graph replays need no new parameters)
   int g, l;
   float ls_trans, ls_rot, T;
@@ -71,6 +73,7 @@ struct ScoreArgs {
 // launchers (return cudaError_t of the launch)
 cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectric, int n_blocks, cudaStream_t st);
 cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st);
+cudaError_t launch_lsk_accept(const ScoreArgs& a, cudaStream_t st);
 // lane mapping for a uniform launch of nseg segments of seg_size poses: sets mixed / bps / fbps;
 // returns the number of scoring blocks
 int plan_uniform(ScoreArgs& a, int seg_size);

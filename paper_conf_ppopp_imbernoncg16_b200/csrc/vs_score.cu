@@ -231,14 +231,15 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
     q = r.q;
     t = r.t;
   } else {
-    j = __ldg(a.J + k * a.m + p);
+    const int jj = p / a.K, kk = p - jj * a.K;
+    j = __ldg(a.J + k * a.m + jj);
     jx = k * a.P + j;
     const PoseRec r = a.poses[jx];
     q = r.q;
     t = r.t;
     old_score = r.t.w;
     perturb(q, t, a.ls_trans, a.ls_rot, a.T, *a.seedp, (uint32_t)j, (uint32_t)spot, (uint32_t)a.g, TAG_LS,
-            2u * (uint32_t)a.l);
+            2u * (uint32_t)(a.l * a.K + kk));
   }
 
   // ---- rotation (homogeneous form, R11)
@@ -301,6 +302,8 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
         const int pidx = a.uniform ? k * a.seg_stride + p : item;
         a.poses[pidx].t.w = score;
         if (a.orig) a.score_out[__ldg(a.orig + pidx)] = score;
+      } else if (a.K > 1) {
+        a.pscore[item] = score;                                  // best of K chosen by lsk_accept_kernel
       } else if (score < old_score) {                            // strict improvement (R16)
         PoseRec rr;
         rr.q = q;
@@ -341,6 +344,8 @@ __global__ void finalize_kernel(const ScoreArgs a, int n_items_blocks) {
     const int pidx = a.uniform ? k * a.seg_stride + p : item;
     a.poses[pidx].t.w = score;
     if (a.orig) a.score_out[__ldg(a.orig + pidx)] = score;
+  } else if (a.K > 1) {
+    a.pscore[item] = score;
   } else {
     const int spot = __ldg(a.seg_spot + k);
     const int j = __ldg(a.J + k * a.m + p);
@@ -389,6 +394,35 @@ cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStre
 }  // namespace vsk
 
 namespace vsk {
+
+// Parallel-neighbourhood Improve (N4): element j of segment k takes the best of its K proposals
+// (strict <, lowest k on ties) if that is strictly better than itself.
+__global__ void lsk_accept_kernel(const ScoreArgs a) {
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= a.nseg * a.m) return;
+  const int k = idx / a.m, jj = idx - k * a.m;
+  const float* ps = a.pscore + ((size_t)k * a.m + jj) * a.K;
+  int best = 0;
+  for (int kk = 1; kk < a.K; ++kk)
+    if (ps[kk] < ps[best]) best = kk;
+  const int j = __ldg(a.J + k * a.m + jj);
+  const int jx = k * a.P + j;
+  PoseRec r = a.poses[jx];
+  if (ps[best] < r.t.w) {
+    float4 q = r.q, t = r.t;
+    perturb(q, t, a.ls_trans, a.ls_rot, a.T, *a.seedp, (uint32_t)j, (uint32_t)__ldg(a.seg_spot + k), (uint32_t)a.g,
+            TAG_LS, 2u * (uint32_t)(a.l * a.K + best));
+    r.q = q;
+    r.t = make_float4(t.x, t.y, t.z, ps[best]);
+    a.poses[jx] = r;
+  }
+}
+
+cudaError_t launch_lsk_accept(const ScoreArgs& a, cudaStream_t st) {
+  const int n = a.nseg * a.m;
+  lsk_accept_kernel<<<(n + 127) / 128, 128, 0, st>>>(a);
+  return cudaGetLastError();
+}
 
 // Lanes = poses (warp-uniform ligand group, H-bond-specialised loop) unless the segment is short
 // enough that (pose, group) items fill clearly more lanes (e.g. Improve's m = 51 or 13 poses).

@@ -40,7 +40,8 @@ class ScoreParams(C.Structure):
 class MHParams(C.Structure):
     _fields_ = [("population", C.c_int), ("generations", C.c_int), ("ls_steps", C.c_int),
                 ("improve_frac", C.c_float), ("p_mut", C.c_float), ("mut_trans", C.c_float),
-                ("mut_rot", C.c_float), ("ls_trans", C.c_float), ("ls_rot", C.c_float)]
+                ("mut_rot", C.c_float), ("ls_trans", C.c_float), ("ls_rot", C.c_float),
+                ("ls_neighbours", C.c_int)]
 
 
 class Stats(C.Structure):

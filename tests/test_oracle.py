@@ -417,3 +417,22 @@ def test_abi_errors(oracle_mod):
     # all-pairs mode accepts any translation
     _, oa = _tiny(oracle_mod, rc=0.0)
     assert np.isfinite(oa.score([0], [[1, 0, 0, 0]], [[30.0, 0, 0]]))[0]
+
+
+def test_parallel_neighbourhood_ls(oracle_mod):
+    """N4: best-of-K proposals per Improve step; K = 1 is plain hill climbing (same streams); never worse."""
+    prob, o = _tiny(oracle_mod)
+    mp1 = oracle_mod.mh_preset(4, population=32)
+    assert mp1.ls_neighbours == 1
+    p0 = o.init_pose(5, 0, 0)
+    np.testing.assert_array_equal(o.ls_proposal(mp1, 5, 0, 0, 3, 7, p0), o.ls_proposal(mp1, 5, 0, 0, 3, 7, p0, k=0))
+    mp4 = oracle_mod.mh_preset(4, population=32, ls_neighbours=4)
+    # proposal k of step l uses counter 2 (l K + k): step 1, k 0 of K = 4 is step 4 of K = 1
+    np.testing.assert_array_equal(o.ls_proposal(mp4, 5, 0, 0, 1, 7, p0, k=0), o.ls_proposal(mp1, 5, 0, 0, 4, 7, p0))
+    _, b0 = o.run(oracle_mod.mh_preset(1, population=32, generations=0), 5)
+    _, b1 = o.run(mp1, 5)
+    _, b4 = o.run(mp4, 5)
+    assert np.all(b1 <= b0) and np.all(b4 <= b0)
+    assert np.mean(b4) <= np.mean(b1) + 1e-9
+    with pytest.raises(oracle_mod.OracleError):
+        o.run(oracle_mod.mh_preset(4, ls_neighbours=0), 5)
