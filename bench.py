@@ -11,8 +11,10 @@ every individual and local-search proposal, selection, on device.
   python bench.py --impl reference ...                      (the fp64 CPU oracle arm)
 
 metric: atom-pair interactions/s (BASELINE.json); a pair = one ligand atom x
-one receptor atom of the spot's streamed list (n_lig x list length per pose;
-SURVEY.md §8(d)).  Poses/s are reported alongside.
+one receptor atom streamed for that pose: the whole receptor
+in all-pairs mode, the inner shells of the spot's distance-sorted cutoff list
+in cutoff mode (atoms farther than R_w + rc are provably out of range and are
+neither streamed nor counted).  Poses/s are reported alongside.
 """
 from __future__ import annotations
 

@@ -94,6 +94,8 @@ struct vs_ctx {
   int* d_iota = nullptr;
   unsigned long long* d_counters = nullptr;
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
+  int* d_shell = nullptr;               // cutoff mode: [n_spots][NSHELL] shell prefix counts
+  int* d_group_natoms = nullptr;        // real atoms per ligand group
   cudaStream_t stream = nullptr;
   cudaStream_t sub[NSUB] = {};          // per-spot-group streams of vs_run
   cudaEvent_t ev_fork = nullptr, ev_join[NSUB] = {};
@@ -167,7 +169,10 @@ ScoreArgs base_args(vs_ctx* c) {
   a.n_chunks = c->n_chunks;
   a.n_lig = c->n_lig;
   a.r2min = c->r2min;
+  a.rc = c->rc;
   a.rc2 = c->rc2;
+  a.shell = c->d_shell;
+  a.group_natoms = c->d_group_natoms;
   a.inv_rc2 = c->inv_rc2;
   a.hbC = c->hbC;
   a.hbD = c->hbD;
@@ -651,7 +656,9 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   std::vector<LigSlot> slots((size_t)c->n_groups * K_SLOTS);
   std::memset(slots.data(), 0, sizeof(LigSlot) * slots.size());
   double rmax = 0.0;
+  std::vector<int> slot_count(c->n_groups, 0);
   auto put = [&](int slot, int i) {
+    slot_count[slot / K_SLOTS]++;
     const int t = lig_type[i];
     LigSlot& s = slots[slot];
     s.lq.x = lig_xyz[3 * i] - cen[0];
@@ -681,6 +688,14 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
       vs_destroy(c);
       return set_err(VS_ERR_INVALID_ARGUMENT, "internal: ligand slot layout");
     }
+  }
+  {
+    // real atoms per group, counted from the placement (an all-zero real atom, e.g. type X at the
+    // centroid, is still counted)
+    std::vector<int> gn(c->n_groups, 0);
+    for (int g = 0; g < c->n_groups; ++g) gn[g] = slot_count[g];
+    CKC(cudaMalloc(&c->d_group_natoms, sizeof(int) * c->n_groups), "alloc");
+    CKC(cudaMemcpy(c->d_group_natoms, gn.data(), sizeof(int) * c->n_groups, cudaMemcpyHostToDevice), "H2D");
   }
   CKC(cudaMalloc(&c->d_lig, sizeof(LigSlot) * slots.size()), "alloc ligand");
   CKC(cudaMemcpy(c->d_lig, slots.data(), sizeof(LigSlot) * slots.size(), cudaMemcpyHostToDevice), "H2D ligand");
@@ -758,6 +773,16 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
     CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, (float)(reach * reach), c->d_list_off, nullptr,
                            c->d_lists, 0, c->stream), "list fill launch");
+    // distance-sorted lists + shell table (per-warp truncation in the scoring kernel)
+    CKT(cudaMemcpyAsync(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
+    RecAtom* sorted = nullptr;
+    CKT(cudaMalloc(&sorted, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
+    CKT(cudaMalloc(&c->d_shell, sizeof(int) * (size_t)n_spots * NSHELL), "alloc shells");
+    cudaError_t es = launch_sort_lists(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_shell, c->stream);
+    if (es == cudaSuccess) es = cudaStreamSynchronize(c->stream);
+    cudaFree(c->d_lists);
+    c->d_lists = sorted;
+    CKT(es, "list sort launch");
   }
   if (!c->d_list_len) CKT(cudaMalloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
   CKT(cudaMemcpy(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
@@ -876,7 +901,7 @@ void vs_destroy(vs_ctx* c) {
   for (auto e : c->ev) cudaEventDestroy(e);
   if (c->gexec) cudaGraphExecDestroy(c->gexec);
   void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_lig, c->d_iota, c->d_counters,
-                  c->d_seed};
+                  c->d_seed, c->d_shell, c->d_group_natoms};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (c->stream) cudaStreamDestroy(c->stream);

@@ -28,6 +28,13 @@ constexpr int NSTAGE = VS_NSTAGE;   // bulk-copy ring depth
 
 enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
 
+// Per-spot lists are sorted by distance from the spot centre; shell[s][b] = number of list atoms with
+// |r| < (b + 1) * SHELL_DR.  A warp whose ligand atoms all lie within R_w of the spot centre streams only
+// the atoms with |r| < R_w + rc (the others are provably beyond the cutoff of every pair).
+constexpr int NSHELL = 256;
+constexpr float SHELL_DR = 0.125f;   // A: table covers 32 A
+constexpr int SORT_MAX = 4096;       // longest list sorted in shared memory (32 KB of keys)
+
 // Work decomposition of one scoring launch: segments (one spot each) of poses,
 // split into 32-pose blocks; blockIdx.y = ligand group chunk.
 struct ScoreArgs {
@@ -36,6 +43,8 @@ struct ScoreArgs {
   const int* list_off;
   const int* list_len;
   const float4* shift;       // added to t + R l (all-pairs: c_s - c0; cutoff: 0)
+  const int* shell;          // cutoff mode: [n_spots][NSHELL] prefix counts of the distance-sorted lists
+  const int* group_natoms;   // real (non-padding) ligand atoms per group, for pair accounting
   const LigSlot* lig;
   int n_groups;              // ligand groups of K_SLOTS slots
   int hb_base, hb_extra;     // group g holds hb_base + (g < hb_extra) H-bond slot pairs, at its end
@@ -43,7 +52,7 @@ struct ScoreArgs {
   int mixed;                 // 1: lanes map to (pose, group) items of a segment (1-warp CTAs, grid.y = 1)
   int n_chunks;              // ceil(n_groups / GROUPS_PER_CTA)
   int n_lig;                 // real ligand atoms (pair accounting)
-  float r2min, rc2, inv_rc2; // rc2 = +inf in all-pairs mode
+  float r2min, rc, rc2, inv_rc2; // rc, rc2 = +inf in all-pairs mode
   float hbC, hbD;
   // segments
   int nseg;
@@ -88,6 +97,9 @@ cudaError_t launch_best(const PoseRec* S, int n_sel, int P, float* best_pose, fl
 cudaError_t launch_build_lists(const float4* rec, const float4* rprm, int n_rec, const float4* spot_c, int n_spots,
                                float reach2, const int* off, int* len, RecAtom* lists, int count_only,
                                cudaStream_t st);
+// sort every cutoff list by distance from its spot centre (stable) and fill the shell table
+cudaError_t launch_sort_lists(RecAtom* lists, RecAtom* tmp, const int* off, const int* len, int n_spots, int* shell,
+                              cudaStream_t st);
 cudaError_t launch_philox(int64_t n, const uint4* ctr, uint2 key, uint4* out, cudaStream_t st);
 // vs_score_poses helpers
 cudaError_t launch_validate(int64_t n, const int32_t* spot, const float* q, const float* t, int n_spots, float T,

@@ -169,6 +169,58 @@ __global__ void list_kernel(const float4* __restrict__ rec, const float4* __rest
   if (threadIdx.x == 0 && count_only) len[s] = base_sh;
 }
 
+// One CTA per spot: (|r|^2, index) keys bitonic-sorted in shared memory, records gathered into tmp
+// in distance order (ties by list position: deterministic), shell prefix counts by binary search.
+// Lists longer than SORT_MAX stay unsorted and get a flat shell table (no truncation).
+__global__ void sort_lists_kernel(const RecAtom* __restrict__ lists, RecAtom* __restrict__ tmp, const int* off,
+                                  const int* len, int* shell) {
+  extern __shared__ uint64_t skeys[];
+  const int s = blockIdx.x;
+  const int n = len[s];
+  const RecAtom* L = lists + off[s];
+  RecAtom* O = tmp + off[s];
+  int* sh = shell + (size_t)s * NSHELL;
+  if (n > SORT_MAX) {
+    for (int i = threadIdx.x; i < n; i += blockDim.x) O[i] = L[i];
+    for (int b = threadIdx.x; b < NSHELL; b += blockDim.x) sh[b] = n;
+    return;
+  }
+  int N = 1;
+  while (N < n) N <<= 1;
+  for (int i = threadIdx.x; i < N; i += blockDim.x) {
+    uint64_t key = ~0ull;
+    if (i < n) {
+      const float4 x = L[i].xq;
+      const float d2 = x.x * x.x + x.y * x.y + x.z * x.z;
+      key = ((uint64_t)__float_as_uint(d2) << 32) | (uint32_t)i;
+    }
+    skeys[i] = key;
+  }
+  __syncthreads();
+  for (int size = 2; size <= N; size <<= 1)
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      for (int i = threadIdx.x; i < (N >> 1); i += blockDim.x) {
+        const int lo = 2 * i - (i & (stride - 1)), hi = lo + stride;
+        const bool asc = (lo & size) == 0;
+        const uint64_t a = skeys[lo], b = skeys[hi];
+        if ((a > b) == asc) { skeys[lo] = b; skeys[hi] = a; }
+      }
+      __syncthreads();
+    }
+  for (int i = threadIdx.x; i < n; i += blockDim.x) O[i] = L[(uint32_t)skeys[i]];
+  // shell[b] = #atoms with |r|^2 < ((b+1) DR)^2  (upper bound search on the sorted d^2)
+  for (int b = threadIdx.x; b < NSHELL; b += blockDim.x) {
+    const float R = (float)(b + 1) * SHELL_DR;
+    const uint32_t lim = __float_as_uint(R * R);
+    int lo = 0, hi = n;
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if ((uint32_t)(skeys[mid] >> 32) < lim) lo = mid + 1; else hi = mid;
+    }
+    sh[b] = lo;
+  }
+}
+
 __global__ void philox_kernel(int64_t n, const uint4* ctr, uint2 key, uint4* out) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) out[i] = philox4x32_10(ctr[i], key);
@@ -276,6 +328,12 @@ cudaError_t launch_build_lists(const float4* rec, const float4* rprm, int n_rec,
                                float reach2, const int* off, int* len, RecAtom* lists, int count_only,
                                cudaStream_t st) {
   list_kernel<<<n_spots, 256, 0, st>>>(rec, rprm, n_rec, spot_c, reach2, off, len, lists, count_only);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_sort_lists(RecAtom* lists, RecAtom* tmp, const int* off, const int* len, int n_spots, int* shell,
+                              cudaStream_t st) {
+  sort_lists_kernel<<<n_spots, 1024, sizeof(uint64_t) * SORT_MAX, st>>>(lists, tmp, off, len, shell);
   return cudaGetLastError();
 }
 

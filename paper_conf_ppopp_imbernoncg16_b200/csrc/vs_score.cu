@@ -259,7 +259,25 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
   const LigSlot* L = a.lig + (size_t)group * K_SLOTS;
 
   // ---- receptor list of the spot through the bulk-copy ring
-  const int off = __ldg(a.list_off + spot), len = __ldg(a.list_len + spot);
+  const int off = __ldg(a.list_off + spot);
+  int len = __ldg(a.list_len + spot);
+  if (CUT && a.shell) {
+    // the list is sorted by |r|: atoms farther than R_w + rc from the spot centre, R_w = max |x_i| over the
+    // warp's ligand atoms, are beyond the cutoff of every pair of this warp -> stream only the inner shells
+    float r2m = 0.0f;
+#pragma unroll
+    for (int sl = 0; sl < K_SLOTS; ++sl) {
+      const float4 l = __ldg(&L[sl].lq);
+      const float x = ox + (R[0] * l.x + R[1] * l.y + R[2] * l.z);
+      const float y = oy + (R[3] * l.x + R[4] * l.y + R[5] * l.z);
+      const float z = oz + (R[6] * l.x + R[7] * l.y + R[8] * l.z);
+      r2m = fmaxf(r2m, x * x + y * y + z * z);
+    }
+    r2m = __uint_as_float(__reduce_max_sync(0xffffffffu, __float_as_uint(r2m)));
+    const float reach = sqrtf(r2m) + a.rc + 0.01f;                 // 0.01 A absorbs fp32 rounding
+    const int b = (int)ceilf(reach * (1.0f / SHELL_DR)) - 1;
+    if (b < NSHELL) len = min(len, __ldg(a.shell + (size_t)spot * NSHELL + max(b, 0)));
+  }
   const RecAtom* src = a.lists + off;
   const int nt = (len + TILE - 1) / TILE;
   if (threadIdx.x == 0) {
@@ -289,6 +307,15 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
     default: e = sweep<K_PAIRS, CUT, DIEL>(a, L, R, ox, oy, oz, tile, full, relcnt, src, len, nt, nwarps); break;
   }
 
+  // pairs evaluated: real ligand atoms of each lane's group x receptor atoms streamed; poses counted once
+  // (by the CTA holding their group-0 item)
+  unsigned npair = active ? (unsigned)__ldg(a.group_natoms + group) : 0u;
+  npair = __reduce_add_sync(0xffffffffu, npair);
+  const unsigned n0 = __popc(__ballot_sync(0xffffffffu, active && group == 0));
+  if (lane == 0 && a.counters) {
+    if (npair) atomicAdd(a.counters + 0, (unsigned long long)npair * (unsigned long long)len);
+    if (n0) atomicAdd(a.counters + 1, (unsigned long long)n0);
+  }
   red[warp][lane] = e;
   __syncthreads();
   if (warp == 0) {
@@ -310,12 +337,6 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
         rr.t = make_float4(t.x, t.y, t.z, score);
         a.poses[jx] = rr;
       }
-    }
-    // poses of this CTA counted once: those whose group 0 item it holds
-    const unsigned n0 = __popc(__ballot_sync(0xffffffffu, active && group == 0));
-    if (lane == 0 && n0 && a.counters) {
-      atomicAdd(a.counters + 0, (unsigned long long)n0 * (unsigned long long)a.n_lig * (unsigned long long)len);
-      atomicAdd(a.counters + 1, (unsigned long long)n0);
     }
   }
 }

@@ -213,17 +213,25 @@ def test_device_entry_point(gpu, oracle_mod):
 
 
 def test_stats_count_pairs(gpu, oracle_mod):
+    """Pairs counted = real ligand atoms x receptor atoms streamed.  All-pairs mode streams the whole receptor;
+    cutoff mode streams each warp's inner shells of the distance-sorted spot list (<= the full list)."""
     prob = synth.make_problem("tiny")
-    g, _ = both(oracle_mod, prob, 12.0)
+    spot, q, t = synth.make_poses(100, 4, 3.0, seed=2)
+    g, _ = both(oracle_mod, prob, 0.0)
     g.reset_stats()
     g.set_timing(True)
-    spot, q, t = synth.make_poses(100, 4, 3.0, seed=2)
     g.score_poses(spot, q, t)
     st = g.stats()
-    lens = g.list_lengths()
-    assert st["poses_scored"] == 100
-    assert st["pairs"] == int(sum(lens[s] for s in spot)) * prob.cfg.n_lig
+    assert st["poses_scored"] == 100 and st["pairs"] == 100 * prob.cfg.n_rec * prob.cfg.n_lig
     assert st["score_launches"] == 1 and st["timed_launches"] == 1 and st["score_ms"] > 0
+    gm = vs.Context.from_problem(synth.make_problem("medium"), vs.score_params(cutoff=12.0))
+    pm = synth.make_problem("medium")
+    spot, q, t = synth.make_poses(4000, pm.cfg.n_spots, 3.0, seed=2)
+    gm.reset_stats()
+    gm.score_poses(spot, q, t)
+    st = gm.stats()
+    full = int(sum(int(gm.list_lengths()[s]) for s in spot)) * pm.cfg.n_lig
+    assert st["poses_scored"] == 4000 and 0.5 * full < st["pairs"] < full     # shells skip ~20-30 %
 
 
 # ------------------------------------------------------------------ metaheuristic
