@@ -67,7 +67,7 @@ struct DevBuf {
 constexpr int NSUB = 4;  // spot groups (streams) of one vs_run
 
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
-           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_COUNT };
+           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_PERM, B_COUNT };
 
 bool finite_arr(const float* p, int64_t n) {
   for (int64_t i = 0; i < n; ++i)
@@ -256,6 +256,7 @@ struct Body {
   int* JJ;
   double* part;
   float* pscore;
+  int* perm;
   float *best_pose, *best_score;
 };
 
@@ -305,6 +306,10 @@ vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, Tra
   if (r != VS_OK) return r;
   ScoreArgs a = q.plain;
   a.poses = q.S;
+  if (a.perm) {
+    CK(launch_popsort(3, q.S, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
+    c->launches++;
+  }
   if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, 0, 0, q.ns, P, q.S)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.S, 0, tr)) != VS_OK) return r;
@@ -325,6 +330,10 @@ vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, int g, Tr
   if (r != VS_OK) return r;
   ScoreArgs a = q.plain;
   a.poses = q.C;
+  if (a.perm) {
+    CK(launch_popsort(3, q.C, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
+    c->launches++;
+  }
   if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, g, 0, q.ns, P, q.C)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.C, g, tr)) != VS_OK) return r;
@@ -364,7 +373,9 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     pl.seg_stride = P;
     pl.P = P;
     pl.partial = b.part ? b.part + (size_t)k0 * std::max(P, m * mp->ls_neighbours) * c->n_chunks : nullptr;
+    pl.perm = (!c->all_pairs && b.perm) ? b.perm + (size_t)k0 * P : nullptr;  // |t| order: tighter shells
     q.ls = pl;
+    q.ls.perm = nullptr;
     plan_uniform(pl, P);
     plan_uniform(q.ls, m * mp->ls_neighbours);
     q.ls.J = q.J;
@@ -415,6 +426,7 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   CK(c->buf[B_J].ensure(sizeof(int) * (size_t)ns * m), "alloc");
   const size_t items = (size_t)ns * std::max(P, m * mp->ls_neighbours);
   if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * items * c->n_chunks), "alloc");
+  CK(c->buf[B_PERM].ensure(sizeof(int) * (size_t)ns * P), "alloc");
   if (mp->ls_neighbours > 1) CK(c->buf[B_PSCORE].ensure(sizeof(float) * (size_t)ns * m * mp->ls_neighbours), "alloc");
   int* seg = (int*)c->buf[B_SEG].p;
   if (spot_ids)
@@ -435,6 +447,7 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   b.JJ = (int*)c->buf[B_J].p;
   b.part = (double*)c->buf[B_PART].p;
   b.pscore = mp->ls_neighbours > 1 ? (float*)c->buf[B_PSCORE].p : nullptr;
+  b.perm = (int*)c->buf[B_PERM].p;
   b.best_pose = d_best_pose;
   b.best_score = d_best_score;
   if (tr || !c->graphs) return enqueue_body(c, b, st, tr);

@@ -66,6 +66,7 @@ struct ScoreArgs {
   PoseRec* poses;            // segment k pose p at k*seg_stride + p (uniform) or pose_prefix[k] + p
   int seg_stride;
   const int* orig;           // optional: original index of each pose -> score_out
+  const int* perm;           // optional (uniform PLAIN): scoring order of segment k, [nseg][seg_size]
   float* score_out;
   double* partial;           // n_chunks > 1: [n_poses_total][n_chunks]
   // LS (Improve step): X[k*P + J[k*m + jj]] perturbed, scored, accepted if better

@@ -72,8 +72,9 @@ __device__ __forceinline__ uint64_t pkey(float score, uint32_t idx) {
   return ((uint64_t)ord_f32(score) << 32) | idx;
 }
 
-// One CTA per spot.  mode 0: J = best m of S by (score, index);
-// mode 1: S_out = S sorted; mode 2: S_out = best P of S ++ C (S first on ties).
+// One CTA per spot.  mode 0: J = best m of S by (score, index) (listed by |t|);
+// mode 1: S_out = S sorted; mode 2: S_out = best P of S ++ C (S first on ties);
+// mode 3: J = the P indices of S ordered by |t| (scoring order).
 __global__ void popsort_kernel(int mode, const PoseRec* __restrict__ S, const PoseRec* __restrict__ C,
                                PoseRec* __restrict__ S_out, int* __restrict__ J, int P, int m, int N) {
   extern __shared__ uint64_t keys[];
@@ -103,8 +104,39 @@ __global__ void popsort_kernel(int mode, const PoseRec* __restrict__ S, const Po
       __syncthreads();
     }
   }
-  if (mode == 0) {
-    for (int r = threadIdx.x; r < m; r += blockDim.x) J[(size_t)k * m + r] = (int)(uint32_t)keys[r];
+  if (mode == 0 || mode == 3) {
+    // mode 0: the best m by (score, index), then re-ordered by distance from the spot centre so that the
+    // scoring warps hold poses of similar |t| (tighter shell truncation; the Improve steps of distinct
+    // elements are independent, so their order does not change any result).
+    // mode 3: all P indices ordered by |t| (scoring order of a population; no result depends on it).
+    const int cnt = mode == 0 ? m : P;
+    __syncthreads();
+    for (int i = threadIdx.x; i < N; i += blockDim.x) {
+      uint64_t key = ~0ull;
+      if (i < cnt) {
+        const uint32_t o = (uint32_t)keys[i];
+        const float4 t = Sk[o].t;
+        key = ((uint64_t)__float_as_uint(t.x * t.x + t.y * t.y + t.z * t.z) << 32) | o;
+      }
+      keys[i] = key;  // same slot read and written by this thread only
+    }
+    __syncthreads();
+    for (int size = 2; size <= N; size <<= 1) {
+      for (int stride = size >> 1; stride > 0; stride >>= 1) {
+        for (int i = threadIdx.x; i < (N >> 1); i += blockDim.x) {
+          const int lo = 2 * i - (i & (stride - 1));
+          const int hi = lo + stride;
+          const bool asc = (lo & size) == 0;
+          const uint64_t a = keys[lo], b = keys[hi];
+          if ((a > b) == asc) {
+            keys[lo] = b;
+            keys[hi] = a;
+          }
+        }
+        __syncthreads();
+      }
+    }
+    for (int r = threadIdx.x; r < cnt; r += blockDim.x) J[(size_t)k * cnt + r] = (int)(uint32_t)keys[r];
   } else {
     for (int r = threadIdx.x; r < P; r += blockDim.x) {
       const int o = (int)(uint32_t)keys[r];

@@ -226,7 +226,7 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
   int jx = 0, j = 0;
   float old_score = 0.0f;
   if (MODE == MODE_PLAIN) {
-    const int pidx = a.uniform ? k * a.seg_stride + p : item;
+    const int pidx = a.uniform ? k * a.seg_stride + (a.perm ? __ldg(a.perm + k * a.seg_size + p) : p) : item;
     const PoseRec r = a.poses[pidx];
     q = r.q;
     t = r.t;
@@ -326,7 +326,7 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
       if (a.n_chunks > 1) {
         a.partial[(size_t)item * a.n_chunks + group] = sum;
       } else if (MODE == MODE_PLAIN) {
-        const int pidx = a.uniform ? k * a.seg_stride + p : item;
+        const int pidx = a.uniform ? k * a.seg_stride + (a.perm ? __ldg(a.perm + k * a.seg_size + p) : p) : item;
         a.poses[pidx].t.w = score;
         if (a.orig) a.score_out[__ldg(a.orig + pidx)] = score;
       } else if (a.K > 1) {
@@ -362,7 +362,7 @@ __global__ void finalize_kernel(const ScoreArgs a, int n_items_blocks) {
   for (int c = 0; c < a.n_chunks; ++c) sum += a.partial[(size_t)item * a.n_chunks + c];
   const float score = (float)sum;
   if (MODE == MODE_PLAIN) {
-    const int pidx = a.uniform ? k * a.seg_stride + p : item;
+    const int pidx = a.uniform ? k * a.seg_stride + (a.perm ? __ldg(a.perm + k * a.seg_size + p) : p) : item;
     a.poses[pidx].t.w = score;
     if (a.orig) a.score_out[__ldg(a.orig + pidx)] = score;
   } else if (a.K > 1) {
