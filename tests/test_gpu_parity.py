@@ -404,3 +404,19 @@ def test_graph_replay_matches_direct_launches(gpu, oracle_mod):
     assert not np.array_equal(r1[1], r2[1])
     st = g.stats()
     assert st["kernel_launches"] > 0 and st["poses_scored"] > 0
+
+
+def test_run_extreme_sizes(gpu, oracle_mod):
+    """Largest population (2048: 4096-key include sort), a 256-atom ligand (43 groups), a single spot, and
+    duplicated spot ids (same global id -> identical results)."""
+    prob = synth.make_custom(900, 256, 3, seed=9)
+    g, o = both(oracle_mod, prob, 12.0)
+    mp_g = vs.mh_preset(3, population=2048, generations=1, ls_steps=1)
+    mp_o = oracle_mod.mh_preset(3, population=2048, generations=1, ls_steps=1)
+    pg, sg = g.run(mp_g, 4, np.array([2], np.int32))
+    po, so = o.run(mp_o, 4, np.array([2], np.int32))
+    assert abs(sg[0] - so[0]) <= 1e-3 * max(abs(so[0]), 1.0)
+    pd, sd = g.run(vs.mh_preset(2, population=16, generations=2), 5, np.array([1, 1, 0, 1], np.int32))
+    np.testing.assert_array_equal(sd[0], sd[1])
+    np.testing.assert_array_equal(sd[0], sd[3])
+    np.testing.assert_array_equal(pd[0], pd[3])
