@@ -380,12 +380,21 @@ def main():
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
+        parts_ms = {"create": 0.0, "run": 0.0, "destroy": 0.0}
         for i in range(n_e2e):
             # sweep: this rank's share of the ligands (static round robin), one context per ligand
             for li in (range(rank, len(ligs), world) if sweep else [0]):
-                with vs.Context(*rec_h, *lig_h[li], spot_h, sp=sp, device=local) as c2:
-                    c2.run(mp, (screen.ligand_seed(args.seed, li) if sweep else args.seed + rank), None)
-                    e2e_ctx_stats.append(c2.stats())
+                ta = time.perf_counter()
+                c2 = vs.Context(*rec_h, *lig_h[li], spot_h, sp=sp, device=local)
+                tb = time.perf_counter()
+                c2.run(mp, (screen.ligand_seed(args.seed, li) if sweep else args.seed + rank), None)
+                tc = time.perf_counter()
+                e2e_ctx_stats.append(c2.stats())
+                c2.close()
+                td = time.perf_counter()
+                parts_ms["create"] += 1e3 * (tb - ta)
+                parts_ms["run"] += 1e3 * (tc - tb)
+                parts_ms["destroy"] += 1e3 * (td - tc)
         dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=cdev)
         e2e_pairs = torch.tensor([sum(s["pairs"] for s in e2e_ctx_stats)], dtype=torch.float64, device=cdev)
         if world > 1:
@@ -395,6 +404,7 @@ def main():
         d2h = n_spots * 8 * 4 * len(ligs)
         e2e = {"value": float(e2e_pairs.item()) / float(dt.item()), "unit": "pairs/s", "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "steps": n_e2e,
+               "ms_per_step_parts": {k: v / n_e2e for k, v in parts_ms.items()},
                "what": "vs_create (receptor/ligand/spot upload + per-spot list build) + vs_run (host spot ids) + "
                        "best poses/scores to host, wall clock" + (", per ligand of the library" if sweep else "")}
 
