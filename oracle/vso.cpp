@@ -231,7 +231,13 @@ double score_pose(const vso_ctx* c, int s, const float qf[4], const float tf[3])
   return total;
 }
 
-bool less_score_index(double sa, int ia, double sb, int ib) { return sa < sb || (sa == sb && ia < ib); }
+// Decisions that the scores take (Improve's accept, the sorts of Select/Include) are made on the scores
+// rounded to fp32, the precision of the kernel (R26); the scores themselves stay fp64.
+float dec(double s) { return (float)s; }
+
+bool less_score_index(double sa, int ia, double sb, int ib) {
+  return dec(sa) < dec(sb) || (dec(sa) == dec(sb) && ia < ib);
+}
 
 // ---------------------------------------------------------------------------
 // Algorithm 1, per spot.
@@ -326,7 +332,7 @@ struct MH {
           Pose cand = X[j];
           perturb(cand, mp.ls_trans, mp.ls_rot, c->T, seed, j, s, g, TAG_LS, 2 * (l * K + k));
           cand.score = score_pose(c, s, cand.q, cand.t);
-          if (cand.score < best.score) best = cand;
+          if (dec(cand.score) < dec(best.score)) best = cand;
         }
         X[j] = best;
       }
@@ -346,7 +352,7 @@ struct MH {
   }
 
   static void sort_by_score(std::vector<Pose>& S) {
-    std::stable_sort(S.begin(), S.end(), [](const Pose& a, const Pose& b) { return a.score < b.score; });
+    std::stable_sort(S.begin(), S.end(), [](const Pose& a, const Pose& b) { return dec(a.score) < dec(b.score); });
   }
 
   Pose run() {
@@ -656,7 +662,7 @@ void vso_include(const double* sS, const double* sC, int32_t P, int32_t* origin)
   std::vector<int> idx(2 * P);
   for (int i = 0; i < 2 * P; ++i) idx[i] = i;
   auto sc = [&](int i) { return i < P ? sS[i] : sC[i - P]; };
-  std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return sc(a) < sc(b); });
+  std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return dec(sc(a)) < dec(sc(b)); });
   for (int k = 0; k < P; ++k) origin[k] = idx[k];
 }
 

@@ -15,7 +15,9 @@
  *     Initialize, End, Select, Combine, Improve, Include -- with the T4
  *     parameters and the Philox streams of DESIGN.md R23.
  * Pose generation uses IEEE fp32 single operations in the written order
- * (reading R24) so that its bytes can be compared with the GPU's.
+ * (reading R24) so that its bytes can be compared with the GPU's; decisions
+ * taken on scores (accept, sorts) compare the fp64 scores rounded to fp32,
+ * the kernel's precision (R26).
  *
  * ABI mirrors include/vs.h with the prefix vso_ (host only).
  */
