@@ -64,7 +64,11 @@ struct DevBuf {
   }
 };
 
-constexpr int NSUB = 4;  // spot groups (streams) of one vs_run
+constexpr int NSUB = 4;       // spot groups (streams) of one vs_run
+constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (plan_uniform)
+#ifndef VS_SPLIT_WARPS
+#define VS_SPLIT_WARPS 16
+#endif
 
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
            B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_PERM, B_COUNT };
@@ -84,6 +88,7 @@ struct vs_ctx {
   int dielectric = 0;
   float T = 3.0f, rc = 0.0f, rc2 = INFINITY, inv_rc2 = 0.0f, r2min = 0.01f, hbC = 0.0f, hbD = 0.0f;
   int n_groups = 0, n_chunks = 1, hb_base = 0, hb_extra = 0;
+  int n_sm = 148;
   std::vector<int> h_list_len;
   int64_t list_total = 0;
   RecAtom* d_lists = nullptr;
@@ -167,6 +172,7 @@ ScoreArgs base_args(vs_ctx* c) {
   a.hb_extra = c->hb_extra;
   a.hb_max = c->hb_base + (c->hb_extra > 0 ? 1 : 0);
   a.n_chunks = c->n_chunks;
+  a.nsplit = 1;
   a.n_lig = c->n_lig;
   a.r2min = c->r2min;
   a.rc = c->rc;
@@ -201,7 +207,7 @@ vs_status score_launch(vs_ctx* c, const ScoreArgs& a, int mode, int n_blocks, cu
   CK(launch_score(a, mode, !c->all_pairs, c->dielectric, n_blocks, st), "score kernel launch");
   c->launches++;
   c->score_launches++;
-  if (a.n_chunks > 1) {
+  if (a.n_chunks * a.nsplit > 1) {
     CK(launch_finalize(a, mode, a.uniform ? a.nseg * a.fbps : n_blocks, st), "finalize kernel launch");
     c->launches++;
   }
@@ -372,12 +378,13 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     pl.uniform = 1;
     pl.seg_stride = P;
     pl.P = P;
-    pl.partial = b.part ? b.part + (size_t)k0 * std::max(P, m * mp->ls_neighbours) * c->n_chunks : nullptr;
+    pl.partial = b.part ? b.part + (size_t)k0 * std::max(P, m * mp->ls_neighbours) * c->n_chunks * MAX_SPLIT : nullptr;
     pl.perm = (!c->all_pairs && b.perm) ? b.perm + (size_t)k0 * P : nullptr;  // |t| order: tighter shells
     q.ls = pl;
     q.ls.perm = nullptr;
-    plan_uniform(pl, P);
-    plan_uniform(q.ls, m * mp->ls_neighbours);
+    const long target = VS_SPLIT_WARPS;  // warps per spot below which the receptor lists are split
+    plan_uniform(pl, P, target);
+    plan_uniform(q.ls, m * mp->ls_neighbours, target);
     q.ls.J = q.J;
     q.ls.m = m;
     q.ls.K = mp->ls_neighbours;
@@ -425,7 +432,7 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   CK(c->buf[B_C].ensure(pop_bytes), "alloc");
   CK(c->buf[B_J].ensure(sizeof(int) * (size_t)ns * m), "alloc");
   const size_t items = (size_t)ns * std::max(P, m * mp->ls_neighbours);
-  if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * items * c->n_chunks), "alloc");
+  CK(c->buf[B_PART].ensure(sizeof(double) * items * c->n_chunks * MAX_SPLIT), "alloc");
   CK(c->buf[B_PERM].ensure(sizeof(int) * (size_t)ns * P), "alloc");
   if (mp->ls_neighbours > 1) CK(c->buf[B_PSCORE].ensure(sizeof(float) * (size_t)ns * m * mp->ls_neighbours), "alloc");
   int* seg = (int*)c->buf[B_SEG].p;
@@ -618,6 +625,11 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   if (!c) return set_err(VS_ERR_OUT_OF_MEMORY, "out of host memory");
   DeviceGuard guard(cuda_device);
   c->dev = cuda_device;
+  {
+    int nsm = 0;
+    if (cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, cuda_device) == cudaSuccess && nsm > 0)
+      c->n_sm = nsm;
+  }
   c->n_rec = n_rec;
   c->n_lig = n_lig;
   c->n_spots = n_spots;

@@ -51,6 +51,7 @@ struct ScoreArgs {
   int hb_max;                // max over groups
   int mixed;                 // 1: lanes map to (pose, group) items of a segment (1-warp CTAs, grid.y = 1)
   int n_chunks;              // ceil(n_groups / GROUPS_PER_CTA)
+  int nsplit;                // receptor-list splits per (pose block, group) (grid.z); partial sums when > 1
   int n_lig;                 // real ligand atoms (pair accounting)
   float r2min, rc, rc2, inv_rc2; // rc, rc2 = +inf in all-pairs mode
   float hbC, hbD;
@@ -86,7 +87,7 @@ cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStre
 cudaError_t launch_lsk_accept(const ScoreArgs& a, cudaStream_t st);
 // lane mapping for a uniform launch of nseg segments of seg_size poses: sets mixed / bps / fbps;
 // returns the number of scoring blocks
-int plan_uniform(ScoreArgs& a, int seg_size);
+int plan_uniform(ScoreArgs& a, int seg_size, long target_warps);
 cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, cudaStream_t st);
 cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, int g,
                            float p_mut, float mut_trans, float mut_rot, float T, cudaStream_t st);

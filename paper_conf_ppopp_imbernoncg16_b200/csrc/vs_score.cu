@@ -278,8 +278,14 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
     const int b = (int)ceilf(reach * (1.0f / SHELL_DR)) - 1;
     if (b < NSHELL) len = min(len, __ldg(a.shell + (size_t)spot * NSHELL + max(b, 0)));
   }
-  const RecAtom* src = a.lists + off;
-  const int nt = (len + TILE - 1) / TILE;
+  // list split (launches too small to fill the GPU): this CTA streams tiles [t0, t1) of the list; the
+  // split partial energies are summed in a fixed order by finalize_kernel
+  const int nt_all = (len + TILE - 1) / TILE;
+  const int t0 = (int)(((long long)nt_all * blockIdx.z) / a.nsplit);
+  const int t1 = (int)(((long long)nt_all * (blockIdx.z + 1)) / a.nsplit);
+  const RecAtom* src = a.lists + off + (size_t)t0 * TILE;
+  len = max(0, min(len, t1 * TILE) - t0 * TILE);
+  const int nt = t1 - t0;
   if (threadIdx.x == 0) {
     for (int s = 0; s < NSTAGE; ++s) {
       mbar_init(&full[s], 1);
@@ -311,7 +317,7 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
   // (by the CTA holding their group-0 item)
   unsigned npair = active ? (unsigned)__ldg(a.group_natoms + group) : 0u;
   npair = __reduce_add_sync(0xffffffffu, npair);
-  const unsigned n0 = __popc(__ballot_sync(0xffffffffu, active && group == 0));
+  const unsigned n0 = __popc(__ballot_sync(0xffffffffu, active && group == 0 && blockIdx.z == 0));
   if (lane == 0 && a.counters) {
     if (npair) atomicAdd(a.counters + 0, (unsigned long long)npair * (unsigned long long)len);
     if (n0) atomicAdd(a.counters + 1, (unsigned long long)n0);
@@ -323,8 +329,8 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
     for (int w = 0; w < nwarps; ++w) sum += red[w][lane];
     const float score = (float)sum;
     if (active) {
-      if (a.n_chunks > 1) {
-        a.partial[(size_t)item * a.n_chunks + group] = sum;
+      if (a.n_chunks * a.nsplit > 1) {
+        a.partial[((size_t)item * a.n_chunks + group) * a.nsplit + blockIdx.z] = sum;
       } else if (MODE == MODE_PLAIN) {
         const int pidx = a.uniform ? k * a.seg_stride + (a.perm ? __ldg(a.perm + k * a.seg_size + p) : p) : item;
         a.poses[pidx].t.w = score;
@@ -359,7 +365,8 @@ __global__ void finalize_kernel(const ScoreArgs a, int n_items_blocks) {
   if (p >= seg_n) return;
   const int item = (a.uniform ? k * a.seg_size : __ldg(a.pose_prefix + k)) + p;
   double sum = 0.0;
-  for (int c = 0; c < a.n_chunks; ++c) sum += a.partial[(size_t)item * a.n_chunks + c];
+  const int np = a.n_chunks * a.nsplit;
+  for (int c = 0; c < np; ++c) sum += a.partial[(size_t)item * np + c];
   const float score = (float)sum;
   if (MODE == MODE_PLAIN) {
     const int pidx = a.uniform ? k * a.seg_stride + (a.perm ? __ldg(a.perm + k * a.seg_size + p) : p) : item;
@@ -395,7 +402,7 @@ static cudaError_t launch_diel(const ScoreArgs& a, int diel, dim3 grid, dim3 blo
 cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectric, int n_blocks, cudaStream_t st) {
   if (n_blocks <= 0) return cudaSuccess;
   const int warps = a.mixed ? 1 : (a.n_chunks > 1 ? GROUPS_PER_CTA : a.n_groups);
-  dim3 grid(n_blocks, a.mixed ? 1 : a.n_chunks), block(warps * 32);
+  dim3 grid(n_blocks, a.mixed ? 1 : a.n_chunks, a.nsplit), block(warps * 32);
   if (mode == MODE_PLAIN)
     return cutoff ? launch_diel<MODE_PLAIN, true>(a, dielectric, grid, block, st)
                   : launch_diel<MODE_PLAIN, false>(a, dielectric, grid, block, st);
@@ -447,7 +454,7 @@ cudaError_t launch_lsk_accept(const ScoreArgs& a, cudaStream_t st) {
 
 // Lanes = poses (warp-uniform ligand group, H-bond-specialised loop) unless the segment is short
 // enough that (pose, group) items fill clearly more lanes (e.g. Improve's m = 51 or 13 poses).
-int plan_uniform(ScoreArgs& a, int seg_size) {
+int plan_uniform(ScoreArgs& a, int seg_size, long target_warps) {  // target: warps per spot
   a.seg_size = seg_size;
   a.fbps = (seg_size + POSES_PER_CTA - 1) / POSES_PER_CTA;
   const long lanes_pose = (long)a.fbps * POSES_PER_CTA * a.n_groups;
@@ -455,6 +462,12 @@ int plan_uniform(ScoreArgs& a, int seg_size) {
   const long lanes_mixed = (items + POSES_PER_CTA - 1) / POSES_PER_CTA * POSES_PER_CTA;
   a.mixed = (GROUPS_PER_CTA == 1 && a.n_groups > 1 && lanes_mixed * 100 < lanes_pose * 95) ? 1 : 0;
   a.bps = a.mixed ? (int)(lanes_mixed / POSES_PER_CTA) : a.fbps;
+  // split each spot's receptor list over up to 8 CTAs when a spot has few warps of work (Improve's m poses,
+  // small populations).  The rule depends only on per-spot quantities, never on how many spots a launch
+  // holds, so results are bitwise independent of the spot chunking and of the number of GPUs.
+  const long warps_per_spot = (long)a.bps * (a.mixed ? 1 : a.n_chunks * GROUPS_PER_CTA);
+  a.nsplit = 1;
+  while (a.nsplit < 8 && warps_per_spot * a.nsplit < target_warps) a.nsplit *= 2;
   return a.bps;
 }
 
