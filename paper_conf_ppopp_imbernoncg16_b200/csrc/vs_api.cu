@@ -3,8 +3,9 @@
 //
 // The paper's host loop copies the candidate set to each GPU and back for
 // every scoring call (Algorithm 2).  Here the whole population
-// lives in HBM for the run; the host only sequences kernel launches on one
-// stream, and the device boundary is crossed at the start (spot ids) and the
+// lives in HBM for the run; the host only sequences kernel launches (spot
+// groups on up to 4 streams, captured as one CUDA graph on repeated calls),
+// and the device boundary is crossed at the start (seed, spot ids) and the
 // end (best pose + score per spot).
 #include <cmath>
 #include <cstdio>
@@ -64,8 +65,14 @@ struct DevBuf {
   }
 };
 
-constexpr int NSUB = 4;       // spot groups (streams) of one vs_run
+#ifndef VS_NSUB
+#define VS_NSUB 4
+#endif
+constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
 constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (plan_uniform)
+#ifndef VS_GROUP_SPOTS
+#define VS_GROUP_SPOTS 16   // spots per stream group at least
+#endif
 #ifndef VS_SPLIT_WARPS
 #define VS_SPLIT_WARPS 16
 #endif
@@ -122,10 +129,12 @@ struct vs_ctx {
 
 namespace {
 
+// A failed allocation leaves the ctx usable (VS_ERR_OUT_OF_MEMORY); any other CUDA error poisons it.
 vs_status cuda_fail(vs_ctx* c, cudaError_t e, const char* where) {
-  if (c) c->poisoned = true;
-  return set_err(e == cudaErrorMemoryAllocation ? VS_ERR_OUT_OF_MEMORY : VS_ERR_CUDA,
-                 std::string(where) + ": " + cudaGetErrorString(e));
+  const bool oom = e == cudaErrorMemoryAllocation;
+  if (oom) cudaGetLastError();  // reset the (non-sticky) last-error state
+  if (c && !oom) c->poisoned = true;
+  return set_err(oom ? VS_ERR_OUT_OF_MEMORY : VS_ERR_CUDA, std::string(where) + ": " + cudaGetErrorString(e));
 }
 
 #define CK(expr, where)                                 \
@@ -357,7 +366,7 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
   // Spots are independent: split them into groups whose generation loops run on separate
   // streams, enqueued generation by generation, so one group's kernels fill the wave tails of
   // another's.
-  const int G = tr ? 1 : std::max(1, std::min(NSUB, ns / 64));
+  const int G = tr ? 1 : std::max(1, std::min(NSUB, ns / VS_GROUP_SPOTS));
   Group grp[NSUB];
   CK(cudaEventRecord(c->ev_fork, st), "event record");
   for (int gi = 0; gi < G; ++gi) {
