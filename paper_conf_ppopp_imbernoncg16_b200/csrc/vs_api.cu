@@ -78,7 +78,7 @@ constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (pla
 #endif
 
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
-           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_PERM, B_COUNT };
+           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_PERM, B_DONE, B_COUNT };
 
 bool finite_arr(const float* p, int64_t n) {
   for (int64_t i = 0; i < n; ++i)
@@ -216,10 +216,6 @@ vs_status score_launch(vs_ctx* c, const ScoreArgs& a, int mode, int n_blocks, cu
   CK(launch_score(a, mode, !c->all_pairs, c->dielectric, n_blocks, st), "score kernel launch");
   c->launches++;
   c->score_launches++;
-  if (a.n_chunks * a.nsplit > 1) {
-    CK(launch_finalize(a, mode, a.uniform ? a.nseg * a.fbps : n_blocks, st), "finalize kernel launch");
-    c->launches++;
-  }
   if (timed) CK(cudaEventRecord(e1, st), "cudaEventRecord");
   return VS_OK;
 }
@@ -234,6 +230,15 @@ vs_status collect_timing(vs_ctx* c) {
   }
   c->ev_used = 0;
   return VS_OK;
+}
+
+// completion counters of split pose energies: zeroed when (re)allocated, kept at zero by the kernels
+cudaError_t ensure_done(vs_ctx* c, size_t items) {
+  const size_t bytes = sizeof(unsigned) * std::max<size_t>(items, 1);
+  if (bytes <= c->buf[B_DONE].cap) return cudaSuccess;
+  cudaError_t e = c->buf[B_DONE].ensure(bytes);
+  if (e == cudaSuccess) e = cudaMemset(c->buf[B_DONE].p, 0, bytes);
+  return e;
 }
 
 struct Tracer {
@@ -272,6 +277,7 @@ struct Body {
   double* part;
   float* pscore;
   int* perm;
+  unsigned* done;
   float *best_pose, *best_score;
 };
 
@@ -388,6 +394,7 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     pl.seg_stride = P;
     pl.P = P;
     pl.partial = b.part ? b.part + (size_t)k0 * std::max(P, m * mp->ls_neighbours) * c->n_chunks * MAX_SPLIT : nullptr;
+    pl.done = b.done + (size_t)k0 * std::max(P, m * mp->ls_neighbours);
     pl.perm = (!c->all_pairs && b.perm) ? b.perm + (size_t)k0 * P : nullptr;  // |t| order: tighter shells
     q.ls = pl;
     q.ls.perm = nullptr;
@@ -442,6 +449,7 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   CK(c->buf[B_J].ensure(sizeof(int) * (size_t)ns * m), "alloc");
   const size_t items = (size_t)ns * std::max(P, m * mp->ls_neighbours);
   CK(c->buf[B_PART].ensure(sizeof(double) * items * c->n_chunks * MAX_SPLIT), "alloc");
+  CK(ensure_done(c, items), "alloc");
   CK(c->buf[B_PERM].ensure(sizeof(int) * (size_t)ns * P), "alloc");
   if (mp->ls_neighbours > 1) CK(c->buf[B_PSCORE].ensure(sizeof(float) * (size_t)ns * m * mp->ls_neighbours), "alloc");
   int* seg = (int*)c->buf[B_SEG].p;
@@ -464,6 +472,7 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   b.part = (double*)c->buf[B_PART].p;
   b.pscore = mp->ls_neighbours > 1 ? (float*)c->buf[B_PSCORE].p : nullptr;
   b.perm = (int*)c->buf[B_PERM].p;
+  b.done = (unsigned*)c->buf[B_DONE].p;
   b.best_pose = d_best_pose;
   b.best_score = d_best_score;
   if (tr || !c->graphs) return enqueue_body(c, b, st, tr);
@@ -519,6 +528,7 @@ vs_status score_device_impl(vs_ctx* c, int64_t n, const int32_t* d_spot, const f
   CK(c->buf[B_SORTED].ensure(sizeof(PoseRec) * n), "alloc");
   CK(c->buf[B_ORIG].ensure(sizeof(int) * n), "alloc");
   if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * n * c->n_chunks), "alloc");
+  CK(ensure_done(c, (size_t)n), "alloc");
   int* valid = (int*)c->buf[B_VALID].p;
   int* counts = (int*)c->buf[B_COUNTS].p;
   int* pp = (int*)c->buf[B_PP].p;
@@ -541,6 +551,7 @@ vs_status score_device_impl(vs_ctx* c, int64_t n, const int32_t* d_spot, const f
   a.orig = orig;
   a.score_out = d_out;
   a.partial = (double*)c->buf[B_PART].p;
+  a.done = (unsigned*)c->buf[B_DONE].p;
   const int64_t blocks = (n + POSES_PER_CTA - 1) / POSES_PER_CTA + ns;
   if (blocks > 0x7fffffff) return set_err(VS_ERR_INVALID_ARGUMENT, "too many poses in one call");
   return score_launch(c, a, MODE_PLAIN, (int)blocks, st);

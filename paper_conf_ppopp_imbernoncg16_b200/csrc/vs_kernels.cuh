@@ -60,7 +60,7 @@ struct ScoreArgs {
   const int* seg_spot;       // [nseg] global spot id
   int uniform;               // 1: every segment has seg_size poses
   int seg_size, bps;         // uniform: poses per segment, scoring blocks per segment
-  int fbps;                  // uniform: 32-pose blocks per segment (finalize)
+  int fbps;                  // uniform: 32-pose blocks per segment
   const int* blk_prefix;     // non-uniform: [nseg+1]
   const int* pose_prefix;    // non-uniform: [nseg+1]
   // PLAIN
@@ -69,7 +69,8 @@ struct ScoreArgs {
   const int* orig;           // optional: original index of each pose -> score_out
   const int* perm;           // optional (uniform PLAIN): scoring order of segment k, [nseg][seg_size]
   float* score_out;
-  double* partial;           // n_chunks > 1: [n_poses_total][n_chunks]
+  double* partial;           // n_chunks * nsplit > 1: [items][n_chunks * nsplit] partial energies
+  unsigned* done;            // [items] contributions received (reset to 0 by the completing CTA)
   // LS (Improve step): X[k*P + J[k*m + jj]] perturbed, scored, accepted if better
   const int* J;
   int m, P;
@@ -83,7 +84,6 @@ struct ScoreArgs {
 
 // launchers (return cudaError_t of the launch)
 cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectric, int n_blocks, cudaStream_t st);
-cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st);
 cudaError_t launch_lsk_accept(const ScoreArgs& a, cudaStream_t st);
 // lane mapping for a uniform launch of nseg segments of seg_size poses: sets mixed / bps / fbps;
 // returns the number of scoring blocks

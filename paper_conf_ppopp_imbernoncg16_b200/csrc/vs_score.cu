@@ -279,7 +279,7 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
     if (b < NSHELL) len = min(len, __ldg(a.shell + (size_t)spot * NSHELL + max(b, 0)));
   }
   // list split (launches too small to fill the GPU): this CTA streams tiles [t0, t1) of the list; the
-  // split partial energies are summed in a fixed order by finalize_kernel
+  // split partial energies are summed in a fixed order by the CTA that completes the pose
   const int nt_all = (len + TILE - 1) / TILE;
   const int t0 = (int)(((long long)nt_all * blockIdx.z) / a.nsplit);
   const int t1 = (int)(((long long)nt_all * (blockIdx.z + 1)) / a.nsplit);
@@ -327,11 +327,26 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
   if (warp == 0) {
     double sum = 0.0;
     for (int w = 0; w < nwarps; ++w) sum += red[w][lane];
+    bool finish = active;
+    if (active && a.n_chunks * a.nsplit > 1) {
+      // the pose's energy is split over ligand groups (and list splits) held by several CTAs: write this
+      // partial; the CTA that completes the pose adds all partials in a fixed order (deterministic) and
+      // applies the epilogue (no separate finalize launch)
+      const int np = a.n_chunks * a.nsplit;
+      const int slot = (a.mixed ? group : chunk) * a.nsplit + blockIdx.z;
+      a.partial[(size_t)item * np + slot] = sum;
+      __threadfence();
+      finish = atomicAdd(a.done + item, 1u) == (unsigned)(np - 1);
+      if (finish) {
+        __threadfence();
+        sum = 0.0;
+        for (int c = 0; c < np; ++c) sum += __ldcg(a.partial + (size_t)item * np + c);
+        a.done[item] = 0u;  // ready for the next launch
+      }
+    }
     const float score = (float)sum;
-    if (active) {
-      if (a.n_chunks * a.nsplit > 1) {
-        a.partial[((size_t)item * a.n_chunks + group) * a.nsplit + blockIdx.z] = sum;
-      } else if (MODE == MODE_PLAIN) {
+    if (finish) {
+      if (MODE == MODE_PLAIN) {
         const int pidx = a.uniform ? k * a.seg_stride + (a.perm ? __ldg(a.perm + k * a.seg_size + p) : p) : item;
         a.poses[pidx].t.w = score;
         if (a.orig) a.score_out[__ldg(a.orig + pidx)] = score;
@@ -343,49 +358,6 @@ __global__ void VS_REGCAP score_kernel(const ScoreArgs a) {
         rr.t = make_float4(t.x, t.y, t.z, score);
         a.poses[jx] = rr;
       }
-    }
-  }
-}
-
-// multi-chunk ligands: fixed-order sum of the chunk partials + the epilogue
-template <int MODE>
-__global__ void finalize_kernel(const ScoreArgs a, int n_items_blocks) {
-  const int bx = blockIdx.x;
-  if (bx >= n_items_blocks) return;
-  if (!a.uniform && bx >= __ldg(a.blk_prefix + a.nseg)) return;
-  int k, blk;
-  if (a.uniform) {  // pose blocks (not the scoring launch's lane blocks)
-    k = bx / a.fbps;
-    blk = bx - k * a.fbps;
-  } else {
-    locate(a, bx, k, blk);
-  }
-  const int seg_n = a.uniform ? a.seg_size : (__ldg(a.pose_prefix + k + 1) - __ldg(a.pose_prefix + k));
-  const int p = blk * POSES_PER_CTA + threadIdx.x;
-  if (p >= seg_n) return;
-  const int item = (a.uniform ? k * a.seg_size : __ldg(a.pose_prefix + k)) + p;
-  double sum = 0.0;
-  const int np = a.n_chunks * a.nsplit;
-  for (int c = 0; c < np; ++c) sum += a.partial[(size_t)item * np + c];
-  const float score = (float)sum;
-  if (MODE == MODE_PLAIN) {
-    const int pidx = a.uniform ? k * a.seg_stride + (a.perm ? __ldg(a.perm + k * a.seg_size + p) : p) : item;
-    a.poses[pidx].t.w = score;
-    if (a.orig) a.score_out[__ldg(a.orig + pidx)] = score;
-  } else if (a.K > 1) {
-    a.pscore[item] = score;
-  } else {
-    const int spot = __ldg(a.seg_spot + k);
-    const int j = __ldg(a.J + k * a.m + p);
-    const int jx = k * a.P + j;
-    PoseRec r = a.poses[jx];
-    if (score < r.t.w) {
-      float4 q = r.q, t = r.t;
-      perturb(q, t, a.ls_trans, a.ls_rot, a.T, *a.seedp, (uint32_t)j, (uint32_t)spot, (uint32_t)a.g, TAG_LS,
-              2u * (uint32_t)a.l);
-      r.q = q;
-      r.t = make_float4(t.x, t.y, t.z, score);
-      a.poses[jx] = r;
     }
   }
 }
@@ -410,14 +382,6 @@ cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectr
                 : launch_diel<MODE_LS, false>(a, dielectric, grid, block, st);
 }
 
-cudaError_t launch_finalize(const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st) {
-  if (n_blocks <= 0) return cudaSuccess;
-  if (mode == MODE_PLAIN)
-    finalize_kernel<MODE_PLAIN><<<n_blocks, POSES_PER_CTA, 0, st>>>(a, n_blocks);
-  else
-    finalize_kernel<MODE_LS><<<n_blocks, POSES_PER_CTA, 0, st>>>(a, n_blocks);
-  return cudaGetLastError();
-}
 
 }  // namespace vsk
 
