@@ -78,7 +78,12 @@ constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (pla
 #endif
 
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
-           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_PERM, B_DONE, B_COUNT };
+           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_PERM, B_DONE, B_PBUF, B_ITEMS, B_E, B_COUNT };
+
+// scoring engines: "cells" (atom-centric chunks + cell-culled list runs, vs_cells.cu) and "poses"
+// (one pose per lane, distance-sorted lists with shell truncation, vs_score.cu); VS_ENGINE=poses selects
+// the latter
+enum Engine { ENGINE_POSES = 0, ENGINE_CELLS = 1 };
 
 bool finite_arr(const float* p, int64_t n) {
   for (int64_t i = 0; i < n; ++i)
@@ -108,6 +113,15 @@ struct vs_ctx {
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
   int* d_shell = nullptr;               // cutoff mode: [n_spots][NSHELL] shell prefix counts
   int* d_group_natoms = nullptr;        // real atoms per ligand group
+  // cells engine
+  int engine = ENGINE_CELLS;
+  int* d_cells = nullptr;               // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
+  float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
+  float4* d_ligx = nullptr;             // [n_lig] centred local coordinates, w = class
+  float4* d_ligp = nullptr;             // [n_lig] es, c12, c6, donor
+  int* d_lig_rank = nullptr;            // [n_lig] rank within the class
+  int nn = 0, nh = 0, H = 0, cn = 0, chb = 0;
+  float W = 0.0f, inv_hm = 0.0f;
   cudaStream_t stream = nullptr;
   cudaStream_t sub[NSUB] = {};          // per-spot-group streams of vs_run
   cudaEvent_t ev_fork = nullptr, ev_join[NSUB] = {};
@@ -123,7 +137,7 @@ struct vs_ctx {
   // CUDA graph of vs_run (captured on the second identical call)
   bool graphs = true, capturing = false, has_last = false;
   cudaGraphExec_t gexec = nullptr;
-  unsigned char gkey[160] = {}, last_key[160] = {};
+  unsigned char gkey[256] = {}, last_key[256] = {};
   uint64_t g_launches = 0, g_score_launches = 0;
 };
 
@@ -241,6 +255,74 @@ cudaError_t ensure_done(vs_ctx* c, size_t items) {
   return e;
 }
 
+// list splits of a cells-engine launch: chunks per spot below VS_SPLIT_WARPS are split over up to MAX_SPLIT
+// list ranges.  Depends only on per-spot quantities (bitwise independence of the spot chunking / GPU count).
+int cell_nsplit(int nch) {
+  int ns = 1;
+  while (ns < MAX_SPLIT && (long)nch * ns < VS_SPLIT_WARPS) ns *= 2;
+  return ns;
+}
+
+CellArgs cell_base(vs_ctx* c) {
+  CellArgs a;
+  std::memset(&a, 0, sizeof(a));
+  a.lists = c->d_lists;
+  a.list_off = c->d_list_off;
+  a.list_len = c->d_list_len;
+  a.cells = c->all_pairs ? nullptr : c->d_cells;
+  a.cR = c->cR;
+  a.ch = c->ch;
+  a.cinv_h = c->cinv_h;
+  a.ligx = c->d_ligx;
+  a.ligp = c->d_ligp;
+  a.lig_rank = c->d_lig_rank;
+  a.n_lig = c->n_lig;
+  a.nn = c->nn;
+  a.nh = c->nh;
+  a.H = c->H;
+  a.cn = c->cn;
+  a.chb = c->chb;
+  a.shift = c->d_shift;
+  a.W = c->W;
+  a.inv_hm = c->inv_hm;
+  a.cut = c->all_pairs ? 0 : 1;
+  a.nsplit = 1;
+  a.K = 1;
+  a.r2min = c->r2min;
+  a.rc = c->rc;
+  a.rc2 = c->rc2;
+  a.inv_rc2 = c->inv_rc2;
+  a.hbC = c->hbC;
+  a.hbD = c->hbD;
+  a.T = c->T;
+  a.counters = c->d_counters;
+  a.seedp = c->d_seed;
+  return a;
+}
+
+vs_status cell_launch(vs_ctx* c, const CellArgs& a, long long n_poses, int nb2, cudaStream_t st) {
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  const bool timed = c->timing && !c->capturing;
+  if (timed) {
+    if (c->ev_used + 2 > c->ev.size()) {
+      for (int i = 0; i < 64; ++i) {
+        cudaEvent_t e;
+        CK(cudaEventCreate(&e), "cudaEventCreate");
+        c->ev.push_back(e);
+      }
+    }
+    e0 = c->ev[c->ev_used];
+    e1 = c->ev[c->ev_used + 1];
+    c->ev_used += 2;
+    CK(cudaEventRecord(e0, st), "cudaEventRecord");
+  }
+  CK(launch_cell_score(a, c->dielectric, n_poses, nb2, st), "cells score launch");
+  c->launches += 3;
+  c->score_launches++;
+  if (timed) CK(cudaEventRecord(e1, st), "cudaEventRecord");
+  return VS_OK;
+}
+
 struct Tracer {
   vs_trace_fn fn = nullptr;
   void* user = nullptr;
@@ -279,9 +361,14 @@ struct Body {
   int* perm;
   unsigned* done;
   float *best_pose, *best_score;
+  // cells engine scratch
+  PoseRec* pbuf;
+  float4* items;
+  double* E;
+  int emax;  // E entries per spot and ligand atom: max over the launches of (poses per spot x list splits)
 };
 
-static_assert(sizeof(Body) <= 160, "graph key storage");
+static_assert(sizeof(Body) <= 256, "graph key storage");
 
 // One group of spots running Algorithm 1 on its own stream.
 struct Group {
@@ -292,6 +379,8 @@ struct Group {
   cudaStream_t st = nullptr;
   ScoreArgs plain, ls;
   int plain_blocks = 0, ls_blocks = 0;
+  CellArgs cplain, cls;                // cells engine
+  int cplain_blocks = 0, cls_blocks = 0;
   bool in_b = false;  // the current population S sits in the second (B) buffer
 };
 
@@ -304,6 +393,15 @@ vs_status improve_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, PoseR
   vs_status r = trace_idx(c, tr, q.st, VS_TRACE_SELECT, g, q.ns, m, q.J);
   if (r != VS_OK) return r;
   for (int l = 0; l < mp->ls_steps; ++l) {
+    if (c->engine == ENGINE_CELLS) {
+      CellArgs a = q.cls;
+      a.poses = X;
+      a.g = g;
+      a.l = l;
+      if ((r = cell_launch(c, a, (long long)q.ns * a.seg_size, q.cls_blocks, q.st)) != VS_OK) return r;
+      if ((r = trace_poses(c, tr, q.st, VS_TRACE_LS, g, l, q.ns, P, X)) != VS_OK) return r;
+      continue;
+    }
     ScoreArgs a = q.ls;
     a.poses = X;
     a.g = g;
@@ -325,13 +423,19 @@ vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, Tra
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_INIT, 0, 0, q.ns, P, q.S);
   if (r != VS_OK) return r;
-  ScoreArgs a = q.plain;
-  a.poses = q.S;
-  if (a.perm) {
-    CK(launch_popsort(3, q.S, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
-    c->launches++;
+  if (c->engine == ENGINE_CELLS) {
+    CellArgs a = q.cplain;
+    a.poses = q.S;
+    if ((r = cell_launch(c, a, (long long)q.ns * P, q.cplain_blocks, q.st)) != VS_OK) return r;
+  } else {
+    ScoreArgs a = q.plain;
+    a.poses = q.S;
+    if (a.perm) {
+      CK(launch_popsort(3, q.S, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
+      c->launches++;
+    }
+    if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   }
-  if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, 0, 0, q.ns, P, q.S)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.S, 0, tr)) != VS_OK) return r;
   CK(launch_popsort(1, q.S, nullptr, q.S2, nullptr, q.ns, P, m, q.st), "sort launch");
@@ -349,13 +453,19 @@ vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, int g, Tr
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_COMBINED, g, 0, q.ns, P, q.C);
   if (r != VS_OK) return r;
-  ScoreArgs a = q.plain;
-  a.poses = q.C;
-  if (a.perm) {
-    CK(launch_popsort(3, q.C, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
-    c->launches++;
+  if (c->engine == ENGINE_CELLS) {
+    CellArgs a = q.cplain;
+    a.poses = q.C;
+    if ((r = cell_launch(c, a, (long long)q.ns * P, q.cplain_blocks, q.st)) != VS_OK) return r;
+  } else {
+    ScoreArgs a = q.plain;
+    a.poses = q.C;
+    if (a.perm) {
+      CK(launch_popsort(3, q.C, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
+      c->launches++;
+    }
+    if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   }
-  if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, g, 0, q.ns, P, q.C)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.C, g, tr)) != VS_OK) return r;
   CK(launch_popsort(2, q.S, q.C, q.S2, nullptr, q.ns, P, m, q.st), "include launch");
@@ -409,6 +519,38 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     q.ls.ls_rot = mp->ls_rot;
     q.plain_blocks = q.ns * pl.bps;
     q.ls_blocks = q.ns * q.ls.bps;
+    if (c->engine == ENGINE_CELLS) {
+      const int mk = m * mp->ls_neighbours, maxpose = std::max(P, mk);
+      CellArgs& cp = q.cplain;
+      cp = cell_base(c);
+      cp.nseg = q.ns;
+      cp.seg_spot = q.seg;
+      cp.uniform = 1;
+      cp.seg_size = P;
+      cp.seg_stride = P;
+      cp.P = P;
+      cp.mode = MODE_PLAIN;
+      cp.nch_u = cell_chunks(P, c->nn, c->nh, c->cn, c->chb);
+      cp.nsplit = cell_nsplit(cp.nch_u);
+      cp.pbuf = b.pbuf + (size_t)k0 * maxpose;
+      cp.items = b.items + (size_t)k0 * maxpose * c->n_lig;
+      cp.E = b.E + (size_t)k0 * c->n_lig * b.emax;
+      cp.E_stride = (long long)q.ns * P * c->n_lig;
+      CellArgs& cl = q.cls;
+      cl = cp;
+      cl.mode = MODE_LS;
+      cl.seg_size = mk;
+      cl.nch_u = cell_chunks(mk, c->nn, c->nh, c->cn, c->chb);
+      cl.nsplit = cell_nsplit(cl.nch_u);
+      cl.E_stride = (long long)q.ns * mk * c->n_lig;
+      cl.J = q.J;
+      cl.m = m;
+      cl.K = mp->ls_neighbours;
+      cl.ls_trans = mp->ls_trans;
+      cl.ls_rot = mp->ls_rot;
+      q.cplain_blocks = q.ns * cp.nch_u * cp.nsplit;
+      q.cls_blocks = q.ns * cl.nch_u * cl.nsplit;
+    }
   }
   vs_status r;
   for (int gi = 0; gi < G; ++gi)
@@ -452,6 +594,17 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   CK(ensure_done(c, items), "alloc");
   CK(c->buf[B_PERM].ensure(sizeof(int) * (size_t)ns * P), "alloc");
   if (mp->ls_neighbours > 1) CK(c->buf[B_PSCORE].ensure(sizeof(float) * (size_t)ns * m * mp->ls_neighbours), "alloc");
+  int emax = 0;
+  if (c->engine == ENGINE_CELLS) {
+    const int mk = m * mp->ls_neighbours, maxpose = std::max(P, mk);
+    if ((long long)ns * maxpose * c->n_lig >= (1ll << 31))
+      return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel x population x n_lig must be < 2^31");
+    emax = P * cell_nsplit(cell_chunks(P, c->nn, c->nh, c->cn, c->chb));
+    if (mp->improve_frac > 0.0f) emax = std::max(emax, mk * cell_nsplit(cell_chunks(mk, c->nn, c->nh, c->cn, c->chb)));
+    CK(c->buf[B_PBUF].ensure(sizeof(PoseRec) * (size_t)ns * maxpose), "alloc");
+    CK(c->buf[B_ITEMS].ensure(sizeof(float4) * (size_t)ns * maxpose * c->n_lig), "alloc");
+    CK(c->buf[B_E].ensure(sizeof(double) * (size_t)ns * c->n_lig * emax), "alloc");
+  }
   int* seg = (int*)c->buf[B_SEG].p;
   if (spot_ids)
     CK(cudaMemcpyAsync(seg, spot_ids, sizeof(int) * ns, cudaMemcpyHostToDevice, st), "H2D spot ids");
@@ -475,6 +628,12 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   b.done = (unsigned*)c->buf[B_DONE].p;
   b.best_pose = d_best_pose;
   b.best_score = d_best_score;
+  if (c->engine == ENGINE_CELLS) {
+    b.pbuf = (PoseRec*)c->buf[B_PBUF].p;
+    b.items = (float4*)c->buf[B_ITEMS].p;
+    b.E = (double*)c->buf[B_E].p;
+    b.emax = emax;
+  }
   if (tr || !c->graphs) return enqueue_body(c, b, st, tr);
 
   // CUDA graph of the whole run: captured on the second identical call, replayed afterwards
@@ -516,9 +675,68 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   return VS_OK;
 }
 
+// cells engine: validate, bucket by spot, then K1-K3 over per-spot segments (slices of <= 2^26 items)
+vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_q, const float* d_t,
+                             float* d_out, cudaStream_t st) {
+  const int ns = c->n_spots;
+  const int64_t slice = std::max<int64_t>(1, (int64_t(1) << 26) / c->n_lig);
+  for (int64_t o = 0; o < n; o += slice) {
+    const int64_t nb = std::min(slice, n - o);
+    const int32_t* sp = d_spot + o;
+    const float* q = d_q + 4 * o;
+    const float* t = d_t + 3 * o;
+    float* out = d_out + o;
+    CK(c->buf[B_VALID].ensure(sizeof(int) * nb), "alloc");
+    CK(c->buf[B_COUNTS].ensure(sizeof(int) * ns), "alloc");
+    CK(c->buf[B_PP].ensure(sizeof(int) * (ns + 1)), "alloc");
+    CK(c->buf[B_BP].ensure(sizeof(int) * (ns + 1)), "alloc");
+    CK(c->buf[B_CUR].ensure(sizeof(int) * ns), "alloc");
+    CK(c->buf[B_SORTED].ensure(sizeof(PoseRec) * nb), "alloc");
+    CK(c->buf[B_ORIG].ensure(sizeof(int) * nb), "alloc");
+    CK(c->buf[B_PBUF].ensure(sizeof(PoseRec) * nb), "alloc");
+    CK(c->buf[B_ITEMS].ensure(sizeof(float4) * nb * c->n_lig), "alloc");
+    CK(c->buf[B_E].ensure(sizeof(double) * nb * c->n_lig), "alloc");
+    int* valid = (int*)c->buf[B_VALID].p;
+    int* counts = (int*)c->buf[B_COUNTS].p;
+    int* pp = (int*)c->buf[B_PP].p;
+    int* cp = (int*)c->buf[B_BP].p;
+    int* cur = (int*)c->buf[B_CUR].p;
+    PoseRec* sorted = (PoseRec*)c->buf[B_SORTED].p;
+    int* orig = (int*)c->buf[B_ORIG].p;
+    CK(cudaMemsetAsync(counts, 0, sizeof(int) * ns, st), "memset");
+    CK(launch_validate(nb, sp, q, t, ns, c->T, c->all_pairs ? 0 : 1, valid, counts, out, st), "validate launch");
+    CK(launch_cell_scan(counts, ns, c->nn, c->nh, c->cn, c->chb, pp, cp, cur, st), "scan launch");
+    CK(launch_scatter(nb, sp, q, t, valid, cur, sorted, orig, st), "scatter launch");
+    c->launches += 3;
+    CellArgs a = cell_base(c);
+    a.nseg = ns;
+    a.seg_spot = c->d_iota;
+    a.uniform = 0;
+    a.pose_prefix = pp;
+    a.chunk_prefix = cp;
+    a.mode = MODE_PLAIN;
+    a.poses = sorted;
+    a.orig = orig;
+    a.score_out = out;
+    a.pbuf = (PoseRec*)c->buf[B_PBUF].p;
+    a.items = (float4*)c->buf[B_ITEMS].p;
+    a.E = (double*)c->buf[B_E].p;
+    a.E_stride = nb * c->n_lig;
+    // pair-kernel grid: an upper bound of sum_k max(ceil(n_k nn / cn), ceil(n_k nh / chb))
+    int64_t blocks = ns;
+    if (c->cn > 0) blocks += (nb * c->nn + c->cn - 1) / c->cn;
+    if (c->chb > 0) blocks += (nb * c->nh + c->chb - 1) / c->chb;
+    if (blocks > 0x7fffffff) return set_err(VS_ERR_INVALID_ARGUMENT, "too many poses in one call");
+    vs_status r = cell_launch(c, a, nb, (int)blocks, st);
+    if (r != VS_OK) return r;
+  }
+  return VS_OK;
+}
+
 vs_status score_device_impl(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_q, const float* d_t,
                             float* d_out, cudaStream_t st) {
   if (n == 0) return VS_OK;
+  if (c->engine == ENGINE_CELLS) return score_device_cells(c, n, d_spot, d_q, d_t, d_out, st);
   const int ns = c->n_spots;
   CK(c->buf[B_VALID].ensure(sizeof(int) * n), "alloc");
   CK(c->buf[B_COUNTS].ensure(sizeof(int) * ns), "alloc");
@@ -744,6 +962,45 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   }
   CKC(cudaMalloc(&c->d_lig, sizeof(LigSlot) * slots.size()), "alloc ligand");
   CKC(cudaMemcpy(c->d_lig, slots.data(), sizeof(LigSlot) * slots.size(), cudaMemcpyHostToDevice), "H2D ligand");
+  {
+    // cells engine: ligand atoms in input order; class 1 = H-bond role (donor / acceptor, R5)
+    const char* ev = std::getenv("VS_ENGINE");
+    c->engine = (ev && std::strcmp(ev, "poses") == 0) ? ENGINE_POSES : ENGINE_CELLS;
+    std::vector<float4> lx(n_lig), lp(n_lig);
+    std::vector<int> rank(n_lig);
+    int cnt[2] = {0, 0};
+    for (int i = 0; i < n_lig; ++i) {
+      const int t = lig_type[i];
+      const int cls = (don[t] != 0.0f || acc[t] != 0.0f) ? 1 : 0;
+      lx[i] = make_float4(lig_xyz[3 * i] - cen[0], lig_xyz[3 * i + 1] - cen[1], lig_xyz[3 * i + 2] - cen[2], (float)cls);
+      const double qk = sp.dielectric == 0 ? (double)sp.coulomb_k * lig_q[i] / 4.0
+                                           : (double)sp.coulomb_k * lig_q[i] / (double)sp.eps_r;
+      lp[i] = make_float4((float)qk, c12[t], c6[t], don[t]);
+      rank[i] = cnt[cls]++;
+    }
+    c->nn = cnt[0];
+    c->nh = cnt[1];
+    // H-bond slot pairs per lane: the launch-uniform H minimising (chunks per pose) x (issue slots per chunk),
+    // with 19 slots per class-0 pair and 23 per H-bond pair
+    double best = 1e300;
+    for (int h = 0; h <= K_PAIRS; ++h) {
+      if ((c->nn > 0 && h == K_PAIRS) || (c->nh > 0 && h == 0)) continue;
+      const double per = std::max(h < K_PAIRS ? c->nn / (64.0 * (K_PAIRS - h)) : 0.0, h > 0 ? c->nh / (64.0 * h) : 0.0);
+      const double cost = per * (19.0 * (K_PAIRS - h) + 23.0 * h);
+      if (cost < best) {
+        best = cost;
+        c->H = h;
+      }
+    }
+    c->cn = 64 * (K_PAIRS - c->H);
+    c->chb = 64 * c->H;
+    CKC(cudaMalloc(&c->d_ligx, sizeof(float4) * n_lig), "alloc ligand");
+    CKC(cudaMalloc(&c->d_ligp, sizeof(float4) * n_lig), "alloc ligand");
+    CKC(cudaMalloc(&c->d_lig_rank, sizeof(int) * n_lig), "alloc ligand");
+    CKC(cudaMemcpy(c->d_ligx, lx.data(), sizeof(float4) * n_lig, cudaMemcpyHostToDevice), "H2D ligand");
+    CKC(cudaMemcpy(c->d_ligp, lp.data(), sizeof(float4) * n_lig, cudaMemcpyHostToDevice), "H2D ligand");
+    CKC(cudaMemcpy(c->d_lig_rank, rank.data(), sizeof(int) * n_lig, cudaMemcpyHostToDevice), "H2D ligand");
+  }
 
   // receptor atoms (absolute) + per-atom parameters
   std::vector<float4> hrec(n_rec), hprm(n_rec);
@@ -818,12 +1075,23 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
     CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, (float)(reach * reach), c->d_list_off, nullptr,
                            c->d_lists, 0, c->stream), "list fill launch");
-    // distance-sorted lists + shell table (per-warp truncation in the scoring kernel)
+    // poses engine: distance-sorted lists + shell table (per-warp truncation in the scoring kernel);
+    // cells engine: cell-sorted lists + cell start table (per-chunk culling)
     CKT(cudaMemcpyAsync(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
     RecAtom* sorted = nullptr;
     CKT(cudaMalloc(&sorted, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
-    CKT(cudaMalloc(&c->d_shell, sizeof(int) * (size_t)n_spots * NSHELL), "alloc shells");
-    cudaError_t es = launch_sort_lists(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_shell, c->stream);
+    cudaError_t es;
+    if (c->engine == ENGINE_CELLS) {
+      c->cR = (float)reach + 0.01f;
+      c->ch = 2.0f * c->cR / (float)CELL_G;
+      c->cinv_h = (float)CELL_G / (2.0f * c->cR);
+      CKT(cudaMalloc(&c->d_cells, sizeof(int) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
+      es = launch_cell_sort(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_cells, c->cR, c->cinv_h,
+                            c->stream);
+    } else {
+      CKT(cudaMalloc(&c->d_shell, sizeof(int) * (size_t)n_spots * NSHELL), "alloc shells");
+      es = launch_sort_lists(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_shell, c->stream);
+    }
     if (es == cudaSuccess) es = cudaStreamSynchronize(c->stream);
     cudaFree(c->d_lists);
     c->d_lists = sorted;
@@ -832,6 +1100,8 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   if (!c->d_list_len) CKT(cudaMalloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
   CKT(cudaMemcpy(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
   CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+  c->W = c->T + (float)rmax + 0.01f;  // cutoff mode: |x_k| <= T + max|l_i| for every transformed atom
+  c->inv_hm = (float)(1 << MORTON_BITS) / (2.0f * c->W);
   CKT(cudaMalloc(&c->d_shift, sizeof(float4) * n_spots), "alloc");
   CKT(cudaMemcpy(c->d_shift, h_shift.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
   CKT(cudaMalloc(&c->d_iota, sizeof(int) * n_spots), "alloc");
@@ -946,7 +1216,7 @@ void vs_destroy(vs_ctx* c) {
   for (auto e : c->ev) cudaEventDestroy(e);
   if (c->gexec) cudaGraphExecDestroy(c->gexec);
   void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_lig, c->d_iota, c->d_counters,
-                  c->d_seed, c->d_shell, c->d_group_natoms};
+                  c->d_seed, c->d_shell, c->d_group_natoms, c->d_cells, c->d_ligx, c->d_ligp, c->d_lig_rank};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (c->stream) cudaStreamDestroy(c->stream);

@@ -82,6 +82,80 @@ struct ScoreArgs {
   unsigned long long* counters;  // [0] pairs, [1] poses
 };
 
+// ---------------------------------------------------------------- "cells" engine (vs_cells.cu)
+// Work unit = chunk of up to CH_ITEMS transformed ligand atoms ("items": one ligand atom of one pose),
+// spatially sorted per spot; the chunk streams only the cell rows of the spot's cell-sorted list
+// within rc of its bounding box.
+constexpr int CELL_G = 24;                         // list grid per spot: G^3 cells over [-R, R]^3
+constexpr int CELL_G3 = CELL_G * CELL_G * CELL_G;
+constexpr int CELL_SORT_MAX = 16384;               // longest list cell-sorted in shared memory (128 KB keys)
+constexpr int CH_ITEMS = 2 * K_PAIRS * 32;         // items per chunk (one warp)
+constexpr int CELL_BATCH = 64;                     // receptor atoms per staging buffer
+constexpr int CELL_MAXRUN = CELL_G * CELL_G;       // one run per cell row at most
+constexpr int MORTON_BITS = 4;                     // item sort grid: 16^3 cells over the spot region
+constexpr int MORTON_BINS = 1 << (3 * MORTON_BITS);
+
+struct CellArgs {
+  // receptor lists (per spot) and the cell start table [n_spots][CELL_G3 + 1] (list positions;
+  // cells[s][0] < 0: list not cell-sorted -> streamed whole)
+  const RecAtom* lists;
+  const int* list_off;
+  const int* list_len;
+  const int* cells;
+  float cR, ch, cinv_h;      // grid half-width (A), cell edge, 1 / edge
+  // ligand (input order)
+  const float4* ligx;        // local x, y, z (centred), w = class (0: no H-bond role, 1: donor / acceptor)
+  const float4* ligp;        // es_i, c12_i, c6_i, donor_i
+  const int* lig_rank;       // rank of the atom within its class
+  int n_lig, nn, nh;         // atoms, of which nn without / nh with an H-bond role
+  int H;                     // H-bond slot pairs per lane (launch-uniform; the first K_PAIRS - H pairs hold class 0)
+  int cn, chb;               // chunk capacities: 64 (K_PAIRS - H) class-0 items, 64 H class-1 items
+  const float4* shift;       // added to t + R l (all-pairs: 0 -- lists are spot-relative)
+  float W, inv_hm;           // item sort grid: [-W, W]^3, 16 cells per axis
+  int cut;                   // cutoff mode (cell culling, spatial item sort)
+  // segments (one spot each)
+  int nseg;
+  const int* seg_spot;
+  int uniform, seg_size;     // uniform: every segment has seg_size poses
+  const int* pose_prefix;    // non-uniform: [nseg + 1]
+  const int* chunk_prefix;   // non-uniform: [nseg + 1]
+  int nch_u;                 // uniform: chunks per segment
+  int nsplit;                // list splits per chunk (partial energies summed by the finalize kernel)
+  // poses
+  int mode;                  // MODE_PLAIN / MODE_LS
+  PoseRec* poses;            // PLAIN: segment k pose p at k * seg_stride + p (uniform) or pose_prefix[k] + p;
+                             // LS: the population X (k * P + j)
+  int seg_stride;
+  const int* orig;           // PLAIN non-uniform: original index of each pose -> score_out
+  float* score_out;
+  const int* J;
+  int m, P, K;
+  const uint64_t* seedp;
+  int g, l;
+  float ls_trans, ls_rot, T;
+  // launch scratch
+  PoseRec* pbuf;             // [launch poses] the pose scored (LS: the proposal, t.w = score of X[j])
+  float4* items;             // [launch items] per segment: class-0 items then class-1 items, each spatially sorted
+  double* E;                 // [nsplit][launch items] per-item energies
+  long long E_stride;
+  float r2min, rc, rc2, inv_rc2;
+  float hbC, hbD;
+  unsigned long long* counters;  // [0] pairs evaluated, [1] poses
+};
+
+__host__ __device__ inline int cell_chunks(int seg_n, int nn, int nh, int cn, int chb) {
+  const long long a = cn > 0 ? ((long long)seg_n * nn + cn - 1) / cn : 0;
+  const long long b = chb > 0 ? ((long long)seg_n * nh + chb - 1) / chb : 0;
+  return (int)(a > b ? a : b);
+}
+
+cudaError_t launch_cell_sort(const RecAtom* lists, RecAtom* out, const int* off, const int* len, int n_spots, int* cells,
+                             float R, float inv_h, cudaStream_t st);
+// K1 + K2 + K3 of one scoring call; n_blocks2 = pair-kernel grid (upper bound when non-uniform)
+cudaError_t launch_cell_score(const CellArgs& a, int dielectric, long long n_poses, int n_blocks2, cudaStream_t st);
+cudaError_t launch_cell_scan(const int* counts, int n, int nn, int nh, int cn, int chb, int* pose_prefix,
+                             int* chunk_prefix, int* cursor, cudaStream_t st);
+
 // launchers (return cudaError_t of the launch)
 cudaError_t launch_score(const ScoreArgs& a, int mode, bool cutoff, int dielectric, int n_blocks, cudaStream_t st);
 cudaError_t launch_lsk_accept(const ScoreArgs& a, cudaStream_t st);

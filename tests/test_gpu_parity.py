@@ -214,7 +214,8 @@ def test_device_entry_point(gpu, oracle_mod):
 
 def test_stats_count_pairs(gpu, oracle_mod):
     """Pairs counted = real ligand atoms x receptor atoms streamed.  All-pairs mode streams the whole receptor;
-    cutoff mode streams each warp's inner shells of the distance-sorted spot list (<= the full list)."""
+    cutoff mode streams a subset of each spot's list (cells engine: the cell rows within rc of each chunk's
+    bounding box; poses engine: each warp's inner shells of the distance-sorted list)."""
     prob = synth.make_problem("tiny")
     spot, q, t = synth.make_poses(100, 4, 3.0, seed=2)
     g, _ = both(oracle_mod, prob, 0.0)
@@ -231,7 +232,26 @@ def test_stats_count_pairs(gpu, oracle_mod):
     gm.score_poses(spot, q, t)
     st = gm.stats()
     full = int(sum(int(gm.list_lengths()[s]) for s in spot)) * pm.cfg.n_lig
-    assert st["poses_scored"] == 4000 and 0.5 * full < st["pairs"] < full     # shells skip ~20-30 %
+    assert st["poses_scored"] == 4000 and 0.25 * full < st["pairs"] < full     # culling skips 30-55 %
+
+
+def test_scores_independent_of_batch_composition(gpu, oracle_mod):
+    """A pose's score depends only on the pose and its spot: scoring it alone, inside a larger batch, or in a
+    shuffled batch gives the same bits (the cells engine sorts each spot's atoms spatially and culls per
+    chunk; out-of-cutoff pairs add exactly zero and in-cutoff pairs are summed in list order)."""
+    prob = synth.make_problem("small")
+    g, o = both(oracle_mod, prob, 12.0)
+    spot, q, t = synth.make_poses(3000, prob.cfg.n_spots, 3.0, seed=11)
+    full = g.score_poses(spot, q, t)
+    perm = np.random.default_rng(3).permutation(3000)
+    shuf = np.empty_like(full)
+    shuf[perm] = g.score_poses(spot[perm], q[perm], t[perm])
+    np.testing.assert_array_equal(full, shuf)
+    sub = np.arange(0, 3000, 7)
+    np.testing.assert_array_equal(full[sub], g.score_poses(spot[sub], q[sub], t[sub]))
+    for i in (0, 1234, 2999):
+        np.testing.assert_array_equal(full[i:i + 1], g.score_poses(spot[i:i + 1], q[i:i + 1], t[i:i + 1]))
+    assert_scores(full[::60], o.score(spot[::60], q[::60], t[::60]))
 
 
 # ------------------------------------------------------------------ metaheuristic
