@@ -722,10 +722,9 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
     a.items = (float4*)c->buf[B_ITEMS].p;
     a.E = (double*)c->buf[B_E].p;
     a.E_stride = nb * c->n_lig;
-    // pair-kernel grid: an upper bound of sum_k max(ceil(n_k nn / cn), ceil(n_k nh / chb))
-    int64_t blocks = ns;
-    if (c->cn > 0) blocks += (nb * c->nn + c->cn - 1) / c->cn;
-    if (c->chb > 0) blocks += (nb * c->nh + c->chb - 1) / c->chb;
+    // pair-kernel grid: an upper bound of sum_k cell_chunks(n_k) (<= n_k n_lig / cn + n_k nh / chb + 3)
+    int64_t blocks = 3 * (int64_t)ns + (nb * c->n_lig) / c->cn + 1;
+    if (c->chb > 0) blocks += (nb * c->nh) / c->chb;
     if (blocks > 0x7fffffff) return set_err(VS_ERR_INVALID_ARGUMENT, "too many poses in one call");
     vs_status r = cell_launch(c, a, nb, (int)blocks, st);
     if (r != VS_OK) return r;
@@ -981,18 +980,19 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     c->nn = cnt[0];
     c->nh = cnt[1];
     // H-bond slot pairs per lane: the launch-uniform H minimising (chunks per pose) x (issue slots per chunk),
-    // with 19 slots per class-0 pair and 23 per H-bond pair
+    // with 19 slots per class-0-only pair and 23 per H-bond pair; class-0 items may overflow
+    // into H-bond slots, so chunks per pose = max(n / CH_ITEMS, nh / (64 H))
     double best = 1e300;
-    for (int h = 0; h <= K_PAIRS; ++h) {
-      if ((c->nn > 0 && h == K_PAIRS) || (c->nh > 0 && h == 0)) continue;
-      const double per = std::max(h < K_PAIRS ? c->nn / (64.0 * (K_PAIRS - h)) : 0.0, h > 0 ? c->nh / (64.0 * h) : 0.0);
-      const double cost = per * (19.0 * (K_PAIRS - h) + 23.0 * h);
-      if (cost < best) {
+    for (int h = 0; h <= CELL_KP; ++h) {
+      if (c->nh > 0 && h == 0) continue;
+      const double per = std::max((double)n_lig / CH_ITEMS, h > 0 ? c->nh / (64.0 * h) : 0.0);
+      const double cost = per * (19.0 * (CELL_KP - h) + 23.0 * h);
+      if (cost < best - 1e-12) {
         best = cost;
         c->H = h;
       }
     }
-    c->cn = 64 * (K_PAIRS - c->H);
+    c->cn = CH_ITEMS;
     c->chb = 64 * c->H;
     CKC(cudaMalloc(&c->d_ligx, sizeof(float4) * n_lig), "alloc ligand");
     CKC(cudaMalloc(&c->d_ligp, sizeof(float4) * n_lig), "alloc ligand");

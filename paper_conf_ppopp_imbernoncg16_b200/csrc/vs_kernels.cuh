@@ -89,8 +89,15 @@ struct ScoreArgs {
 constexpr int CELL_G = 24;                         // list grid per spot: G^3 cells over [-R, R]^3
 constexpr int CELL_G3 = CELL_G * CELL_G * CELL_G;
 constexpr int CELL_SORT_MAX = 16384;               // longest list cell-sorted in shared memory (128 KB keys)
-constexpr int CH_ITEMS = 2 * K_PAIRS * 32;         // items per chunk (one warp)
-constexpr int CELL_BATCH = 64;                     // receptor atoms per staging buffer
+#ifndef VS_CELL_KP
+#define VS_CELL_KP 2
+#endif
+constexpr int CELL_KP = VS_CELL_KP;                // packed float2 item pairs per lane (register blocking)
+constexpr int CH_ITEMS = 2 * CELL_KP * 32;         // items per chunk (one warp)
+#ifndef VS_CELL_BATCH
+#define VS_CELL_BATCH 64
+#endif
+constexpr int CELL_BATCH = VS_CELL_BATCH;          // receptor atoms per staging buffer (2 per lane per 64)
 constexpr int CELL_MAXRUN = CELL_G * CELL_G;       // one run per cell row at most
 constexpr int MORTON_BITS = 4;                     // item sort grid: 16^3 cells over the spot region
 constexpr int MORTON_BINS = 1 << (3 * MORTON_BITS);
@@ -108,8 +115,8 @@ struct CellArgs {
   const float4* ligp;        // es_i, c12_i, c6_i, donor_i
   const int* lig_rank;       // rank of the atom within its class
   int n_lig, nn, nh;         // atoms, of which nn without / nh with an H-bond role
-  int H;                     // H-bond slot pairs per lane (launch-uniform; the first K_PAIRS - H pairs hold class 0)
-  int cn, chb;               // chunk capacities: 64 (K_PAIRS - H) class-0 items, 64 H class-1 items
+  int H;                     // H-bond slot pairs per lane (launch-uniform; the first CELL_KP - H pairs hold class 0 only)
+  int cn, chb;               // chunk capacities: cn = CH_ITEMS items in all, chb = 64 H class-1 items
   const float4* shift;       // added to t + R l (all-pairs: 0 -- lists are spot-relative)
   float W, inv_hm;           // item sort grid: [-W, W]^3, 16 cells per axis
   int cut;                   // cutoff mode (cell culling, spatial item sort)
@@ -143,10 +150,16 @@ struct CellArgs {
   unsigned long long* counters;  // [0] pairs evaluated, [1] poses
 };
 
-__host__ __device__ inline int cell_chunks(int seg_n, int nn, int nh, int cn, int chb) {
-  const long long a = cn > 0 ? ((long long)seg_n * nn + cn - 1) / cn : 0;
-  const long long b = chb > 0 ? ((long long)seg_n * nh + chb - 1) / chb : 0;
-  return (int)(a > b ? a : b);
+// Chunks of a segment of seg_n poses: class-1 items (H-bond role) fill at most cap1 = 64 H slots (the last H
+// slot pairs of each lane), class-0 items the other slots and any H-bond slot left over; a chunk takes the
+// same spatial quantile of both classes, so it must hold ceil(Nn / c) + ceil(Nh / c) <= cap items.
+__host__ __device__ inline int cell_chunks(int seg_n, int nn, int nh, int cap, int cap1) {
+  if (seg_n <= 0) return 0;
+  const long long Nn = (long long)seg_n * nn, Nh = (long long)seg_n * nh;
+  long long c = (Nn + Nh + cap - 1) / cap;
+  if (Nh > 0) c = c > (Nh + cap1 - 1) / cap1 ? c : (Nh + cap1 - 1) / cap1;
+  while ((Nn + c - 1) / c + (Nh + c - 1) / c > cap || (Nh + c - 1) / c > cap1) ++c;
+  return (int)c;
 }
 
 cudaError_t launch_cell_sort(const RecAtom* lists, RecAtom* out, const int* off, const int* len, int n_spots, int* cells,

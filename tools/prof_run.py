@@ -1,0 +1,37 @@
+#!/usr/bin/env python
+"""Profiling driver: one vs_run of a config (direct launches) for ncu, e.g.
+
+  VS_GRAPHS=0 ncu --set full -k regex:cell_pair_kernel -c 2 -o gpurun_out/pair python tools/prof_run.py --generations 1
+
+Runs one warm-up call first when --warm is given (so that lazy module loading is outside the capture).
+"""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="medium")
+    ap.add_argument("--preset", type=int, default=3)
+    ap.add_argument("--generations", type=int, default=1)
+    ap.add_argument("--score-poses", type=int, default=0, help="also score N random poses via vs_score_poses")
+    args = ap.parse_args()
+    import torch
+    from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
+    prob = synth.make_problem(args.config)
+    g = vs.Context.from_problem(prob, vs.score_params(), device=0)
+    mp = vs.mh_preset(args.preset, population=prob.cfg.population, generations=args.generations)
+    g.run(mp, 42)
+    if args.score_poses:
+        spot, q, t = synth.make_poses(args.score_poses, prob.cfg.n_spots, 3.0, seed=1)
+        g.score_poses(spot, q, t)
+    torch.cuda.synchronize()
+    print(g.stats())
+
+
+if __name__ == "__main__":
+    main()
