@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define VS_ABI_VERSION 2
+#define VS_ABI_VERSION 3
 
 #if defined(__GNUC__)
 #define VS_API __attribute__((visibility("default")))
@@ -162,9 +162,11 @@ typedef struct {
   uint64_t kernel_launches;  /* all kernels this ctx launched */
   uint64_t score_launches;   /* scoring-kernel launches (plain + fused local search) */
   uint64_t poses_scored;     /* poses scored (incl. local-search proposals) */
-  uint64_t pairs;            /* algorithmic atom pairs: n_lig x list length per scored pose */
+  uint64_t pairs;            /* workload atom pairs: n_lig x list length (n_rec in all-pairs mode) per scored pose */
   double score_ms;           /* summed CUDA-event time of scoring launches (timing enabled) */
   uint64_t timed_launches;   /* launches covered by score_ms */
+  uint64_t pairs_evaluated;  /* pairs the pair kernel evaluated: item slots x receptor atoms streamed per chunk
+                                (<= pairs in cutoff mode: cell culling skips list atoms beyond rc of a chunk) */
 } vs_stats;
 
 /* enable = 1: bracket every scoring launch with CUDA events on its stream. */

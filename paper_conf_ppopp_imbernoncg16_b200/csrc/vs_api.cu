@@ -69,7 +69,7 @@ struct DevBuf {
 #define VS_NSUB 4
 #endif
 constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
-constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (plan_uniform)
+constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (cell_nsplit)
 #ifndef VS_GROUP_SPOTS
 #define VS_GROUP_SPOTS 16   // spots per stream group at least
 #endif
@@ -77,13 +77,8 @@ constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (pla
 #define VS_SPLIT_WARPS 16
 #endif
 
-enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_PART, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
-           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PSCORE, B_PERM, B_DONE, B_PBUF, B_ITEMS, B_E, B_COUNT };
-
-// scoring engines: "cells" (atom-centric chunks + cell-culled list runs, vs_cells.cu) and "poses"
-// (one pose per lane, distance-sorted lists with shell truncation, vs_score.cu); VS_ENGINE=poses selects
-// the latter
-enum Engine { ENGINE_POSES = 0, ENGINE_CELLS = 1 };
+enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
+           B_SORTED, B_ORIG, B_BEST, B_BESTS, B_PBUF, B_ITEMS, B_E, B_COUNT };
 
 bool finite_arr(const float* p, int64_t n) {
   for (int64_t i = 0; i < n; ++i)
@@ -99,7 +94,6 @@ struct vs_ctx {
   bool all_pairs = false;
   int dielectric = 0;
   float T = 3.0f, rc = 0.0f, rc2 = INFINITY, inv_rc2 = 0.0f, r2min = 0.01f, hbC = 0.0f, hbD = 0.0f;
-  int n_groups = 0, n_chunks = 1, hb_base = 0, hb_extra = 0;
   int n_sm = 148;
   std::vector<int> h_list_len;
   int64_t list_total = 0;
@@ -107,14 +101,9 @@ struct vs_ctx {
   int* d_list_off = nullptr;
   int* d_list_len = nullptr;
   float4* d_shift = nullptr;
-  LigSlot* d_lig = nullptr;
   int* d_iota = nullptr;
-  unsigned long long* d_counters = nullptr;
+  unsigned long long* d_counters = nullptr;  // [0] pairs evaluated, [1] poses, [2] workload pairs
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
-  int* d_shell = nullptr;               // cutoff mode: [n_spots][NSHELL] shell prefix counts
-  int* d_group_natoms = nullptr;        // real atoms per ligand group
-  // cells engine
-  int engine = ENGINE_CELLS;
   int* d_cells = nullptr;               // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
   float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
   float4* d_ligx = nullptr;             // [n_lig] centred local coordinates, w = class
@@ -182,58 +171,6 @@ int improve_count(const vs_mh_params* mp) {
   return (int)m;
 }
 
-ScoreArgs base_args(vs_ctx* c) {
-  ScoreArgs a;
-  std::memset(&a, 0, sizeof(a));
-  a.lists = c->d_lists;
-  a.list_off = c->d_list_off;
-  a.list_len = c->d_list_len;
-  a.shift = c->d_shift;
-  a.lig = c->d_lig;
-  a.n_groups = c->n_groups;
-  a.hb_base = c->hb_base;
-  a.hb_extra = c->hb_extra;
-  a.hb_max = c->hb_base + (c->hb_extra > 0 ? 1 : 0);
-  a.n_chunks = c->n_chunks;
-  a.nsplit = 1;
-  a.n_lig = c->n_lig;
-  a.r2min = c->r2min;
-  a.rc = c->rc;
-  a.rc2 = c->rc2;
-  a.shell = c->d_shell;
-  a.group_natoms = c->d_group_natoms;
-  a.inv_rc2 = c->inv_rc2;
-  a.hbC = c->hbC;
-  a.hbD = c->hbD;
-  a.T = c->T;
-  a.counters = c->d_counters;
-  a.seedp = c->d_seed;
-  return a;
-}
-
-vs_status score_launch(vs_ctx* c, const ScoreArgs& a, int mode, int n_blocks, cudaStream_t st) {
-  cudaEvent_t e0 = nullptr, e1 = nullptr;
-  const bool timed = c->timing && !c->capturing;  // graph replays are timed by the caller as a whole
-  if (timed) {
-    if (c->ev_used + 2 > c->ev.size()) {
-      for (int i = 0; i < 64; ++i) {
-        cudaEvent_t e;
-        CK(cudaEventCreate(&e), "cudaEventCreate");
-        c->ev.push_back(e);
-      }
-    }
-    e0 = c->ev[c->ev_used];
-    e1 = c->ev[c->ev_used + 1];
-    c->ev_used += 2;
-    CK(cudaEventRecord(e0, st), "cudaEventRecord");
-  }
-  CK(launch_score(a, mode, !c->all_pairs, c->dielectric, n_blocks, st), "score kernel launch");
-  c->launches++;
-  c->score_launches++;
-  if (timed) CK(cudaEventRecord(e1, st), "cudaEventRecord");
-  return VS_OK;
-}
-
 vs_status collect_timing(vs_ctx* c) {
   for (size_t i = 0; i + 1 < c->ev_used; i += 2) {
     float ms = 0.0f;
@@ -246,16 +183,7 @@ vs_status collect_timing(vs_ctx* c) {
   return VS_OK;
 }
 
-// completion counters of split pose energies: zeroed when (re)allocated, kept at zero by the kernels
-cudaError_t ensure_done(vs_ctx* c, size_t items) {
-  const size_t bytes = sizeof(unsigned) * std::max<size_t>(items, 1);
-  if (bytes <= c->buf[B_DONE].cap) return cudaSuccess;
-  cudaError_t e = c->buf[B_DONE].ensure(bytes);
-  if (e == cudaSuccess) e = cudaMemset(c->buf[B_DONE].p, 0, bytes);
-  return e;
-}
-
-// list splits of a cells-engine launch: chunks per spot below VS_SPLIT_WARPS are split over up to MAX_SPLIT
+// list splits of a scoring launch: chunks per spot below VS_SPLIT_WARPS are split over up to MAX_SPLIT
 // list ranges.  Depends only on per-spot quantities (bitwise independence of the spot chunking / GPU count).
 int cell_nsplit(int nch) {
   int ns = 1;
@@ -356,12 +284,8 @@ struct Body {
   int* seg;
   PoseRec *SA, *SB, *CC;
   int* JJ;
-  double* part;
-  float* pscore;
-  int* perm;
-  unsigned* done;
   float *best_pose, *best_score;
-  // cells engine scratch
+  // scoring scratch
   PoseRec* pbuf;
   float4* items;
   double* E;
@@ -377,9 +301,7 @@ struct Group {
   PoseRec *S = nullptr, *S2 = nullptr, *C = nullptr;
   int* J = nullptr;
   cudaStream_t st = nullptr;
-  ScoreArgs plain, ls;
-  int plain_blocks = 0, ls_blocks = 0;
-  CellArgs cplain, cls;                // cells engine
+  CellArgs cplain, cls;                // scoring launches: plain (a whole population) and Improve (LS)
   int cplain_blocks = 0, cls_blocks = 0;
   bool in_b = false;  // the current population S sits in the second (B) buffer
 };
@@ -393,24 +315,11 @@ vs_status improve_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, PoseR
   vs_status r = trace_idx(c, tr, q.st, VS_TRACE_SELECT, g, q.ns, m, q.J);
   if (r != VS_OK) return r;
   for (int l = 0; l < mp->ls_steps; ++l) {
-    if (c->engine == ENGINE_CELLS) {
-      CellArgs a = q.cls;
-      a.poses = X;
-      a.g = g;
-      a.l = l;
-      if ((r = cell_launch(c, a, (long long)q.ns * a.seg_size, q.cls_blocks, q.st)) != VS_OK) return r;
-      if ((r = trace_poses(c, tr, q.st, VS_TRACE_LS, g, l, q.ns, P, X)) != VS_OK) return r;
-      continue;
-    }
-    ScoreArgs a = q.ls;
+    CellArgs a = q.cls;
     a.poses = X;
     a.g = g;
     a.l = l;
-    if ((r = score_launch(c, a, MODE_LS, q.ls_blocks, q.st)) != VS_OK) return r;
-    if (a.K > 1) {
-      CK(launch_lsk_accept(a, q.st), "accept launch");
-      c->launches++;
-    }
+    if ((r = cell_launch(c, a, (long long)q.ns * a.seg_size, q.cls_blocks, q.st)) != VS_OK) return r;
     if ((r = trace_poses(c, tr, q.st, VS_TRACE_LS, g, l, q.ns, P, X)) != VS_OK) return r;
   }
   return VS_OK;
@@ -423,18 +332,10 @@ vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, Tra
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_INIT, 0, 0, q.ns, P, q.S);
   if (r != VS_OK) return r;
-  if (c->engine == ENGINE_CELLS) {
+  {
     CellArgs a = q.cplain;
     a.poses = q.S;
     if ((r = cell_launch(c, a, (long long)q.ns * P, q.cplain_blocks, q.st)) != VS_OK) return r;
-  } else {
-    ScoreArgs a = q.plain;
-    a.poses = q.S;
-    if (a.perm) {
-      CK(launch_popsort(3, q.S, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
-      c->launches++;
-    }
-    if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   }
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, 0, 0, q.ns, P, q.S)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.S, 0, tr)) != VS_OK) return r;
@@ -453,18 +354,10 @@ vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, int g, Tr
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_COMBINED, g, 0, q.ns, P, q.C);
   if (r != VS_OK) return r;
-  if (c->engine == ENGINE_CELLS) {
+  {
     CellArgs a = q.cplain;
     a.poses = q.C;
     if ((r = cell_launch(c, a, (long long)q.ns * P, q.cplain_blocks, q.st)) != VS_OK) return r;
-  } else {
-    ScoreArgs a = q.plain;
-    a.poses = q.C;
-    if (a.perm) {
-      CK(launch_popsort(3, q.C, nullptr, nullptr, (int*)a.perm, q.ns, P, 0, q.st), "order launch");
-      c->launches++;
-    }
-    if ((r = score_launch(c, a, MODE_PLAIN, q.plain_blocks, q.st)) != VS_OK) return r;
   }
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, g, 0, q.ns, P, q.C)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.C, g, tr)) != VS_OK) return r;
@@ -496,30 +389,7 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     q.J = b.JJ + (size_t)k0 * m;
     q.st = G > 1 ? c->sub[gi] : st;
     if (G > 1) CK(cudaStreamWaitEvent(q.st, c->ev_fork, 0), "stream wait");
-    ScoreArgs& pl = q.plain;
-    pl = base_args(c);
-    pl.nseg = q.ns;
-    pl.seg_spot = q.seg;
-    pl.uniform = 1;
-    pl.seg_stride = P;
-    pl.P = P;
-    pl.partial = b.part ? b.part + (size_t)k0 * std::max(P, m * mp->ls_neighbours) * c->n_chunks * MAX_SPLIT : nullptr;
-    pl.done = b.done + (size_t)k0 * std::max(P, m * mp->ls_neighbours);
-    pl.perm = (!c->all_pairs && b.perm) ? b.perm + (size_t)k0 * P : nullptr;  // |t| order: tighter shells
-    q.ls = pl;
-    q.ls.perm = nullptr;
-    const long target = VS_SPLIT_WARPS;  // warps per spot below which the receptor lists are split
-    plan_uniform(pl, P, target);
-    plan_uniform(q.ls, m * mp->ls_neighbours, target);
-    q.ls.J = q.J;
-    q.ls.m = m;
-    q.ls.K = mp->ls_neighbours;
-    q.ls.pscore = b.pscore ? b.pscore + (size_t)k0 * m * mp->ls_neighbours : nullptr;
-    q.ls.ls_trans = mp->ls_trans;
-    q.ls.ls_rot = mp->ls_rot;
-    q.plain_blocks = q.ns * pl.bps;
-    q.ls_blocks = q.ns * q.ls.bps;
-    if (c->engine == ENGINE_CELLS) {
+    {
       const int mk = m * mp->ls_neighbours, maxpose = std::max(P, mk);
       CellArgs& cp = q.cplain;
       cp = cell_base(c);
@@ -589,13 +459,8 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   CK(c->buf[B_SB].ensure(pop_bytes), "alloc");
   CK(c->buf[B_C].ensure(pop_bytes), "alloc");
   CK(c->buf[B_J].ensure(sizeof(int) * (size_t)ns * m), "alloc");
-  const size_t items = (size_t)ns * std::max(P, m * mp->ls_neighbours);
-  CK(c->buf[B_PART].ensure(sizeof(double) * items * c->n_chunks * MAX_SPLIT), "alloc");
-  CK(ensure_done(c, items), "alloc");
-  CK(c->buf[B_PERM].ensure(sizeof(int) * (size_t)ns * P), "alloc");
-  if (mp->ls_neighbours > 1) CK(c->buf[B_PSCORE].ensure(sizeof(float) * (size_t)ns * m * mp->ls_neighbours), "alloc");
   int emax = 0;
-  if (c->engine == ENGINE_CELLS) {
+  {
     const int mk = m * mp->ls_neighbours, maxpose = std::max(P, mk);
     if ((long long)ns * maxpose * c->n_lig >= (1ll << 31))
       return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel x population x n_lig must be < 2^31");
@@ -622,13 +487,9 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   b.SB = (PoseRec*)c->buf[B_SB].p;
   b.CC = (PoseRec*)c->buf[B_C].p;
   b.JJ = (int*)c->buf[B_J].p;
-  b.part = (double*)c->buf[B_PART].p;
-  b.pscore = mp->ls_neighbours > 1 ? (float*)c->buf[B_PSCORE].p : nullptr;
-  b.perm = (int*)c->buf[B_PERM].p;
-  b.done = (unsigned*)c->buf[B_DONE].p;
   b.best_pose = d_best_pose;
   b.best_score = d_best_score;
-  if (c->engine == ENGINE_CELLS) {
+  {
     b.pbuf = (PoseRec*)c->buf[B_PBUF].p;
     b.items = (float4*)c->buf[B_ITEMS].p;
     b.E = (double*)c->buf[B_E].p;
@@ -675,7 +536,7 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
   return VS_OK;
 }
 
-// cells engine: validate, bucket by spot, then K1-K3 over per-spot segments (slices of <= 2^26 items)
+// validate, bucket by spot, then K1-K3 over per-spot segments (slices of <= 2^26 items)
 vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_q, const float* d_t,
                              float* d_out, cudaStream_t st) {
   const int ns = c->n_spots;
@@ -735,43 +596,7 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
 vs_status score_device_impl(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_q, const float* d_t,
                             float* d_out, cudaStream_t st) {
   if (n == 0) return VS_OK;
-  if (c->engine == ENGINE_CELLS) return score_device_cells(c, n, d_spot, d_q, d_t, d_out, st);
-  const int ns = c->n_spots;
-  CK(c->buf[B_VALID].ensure(sizeof(int) * n), "alloc");
-  CK(c->buf[B_COUNTS].ensure(sizeof(int) * ns), "alloc");
-  CK(c->buf[B_PP].ensure(sizeof(int) * (ns + 1)), "alloc");
-  CK(c->buf[B_BP].ensure(sizeof(int) * (ns + 1)), "alloc");
-  CK(c->buf[B_CUR].ensure(sizeof(int) * ns), "alloc");
-  CK(c->buf[B_SORTED].ensure(sizeof(PoseRec) * n), "alloc");
-  CK(c->buf[B_ORIG].ensure(sizeof(int) * n), "alloc");
-  if (c->n_chunks > 1) CK(c->buf[B_PART].ensure(sizeof(double) * n * c->n_chunks), "alloc");
-  CK(ensure_done(c, (size_t)n), "alloc");
-  int* valid = (int*)c->buf[B_VALID].p;
-  int* counts = (int*)c->buf[B_COUNTS].p;
-  int* pp = (int*)c->buf[B_PP].p;
-  int* bp = (int*)c->buf[B_BP].p;
-  int* cur = (int*)c->buf[B_CUR].p;
-  PoseRec* sorted = (PoseRec*)c->buf[B_SORTED].p;
-  int* orig = (int*)c->buf[B_ORIG].p;
-  CK(cudaMemsetAsync(counts, 0, sizeof(int) * ns, st), "memset");
-  CK(launch_validate(n, d_spot, d_q, d_t, ns, c->T, c->all_pairs ? 0 : 1, valid, counts, d_out, st), "validate launch");
-  CK(launch_scan(counts, ns, pp, bp, cur, st), "scan launch");
-  CK(launch_scatter(n, d_spot, d_q, d_t, valid, cur, sorted, orig, st), "scatter launch");
-  c->launches += 3;
-  ScoreArgs a = base_args(c);
-  a.nseg = ns;
-  a.seg_spot = c->d_iota;
-  a.uniform = 0;
-  a.blk_prefix = bp;
-  a.pose_prefix = pp;
-  a.poses = sorted;
-  a.orig = orig;
-  a.score_out = d_out;
-  a.partial = (double*)c->buf[B_PART].p;
-  a.done = (unsigned*)c->buf[B_DONE].p;
-  const int64_t blocks = (n + POSES_PER_CTA - 1) / POSES_PER_CTA + ns;
-  if (blocks > 0x7fffffff) return set_err(VS_ERR_INVALID_ARGUMENT, "too many poses in one call");
-  return score_launch(c, a, MODE_PLAIN, (int)blocks, st);
+  return score_device_cells(c, n, d_spot, d_q, d_t, d_out, st);
 }
 
 }  // namespace
@@ -896,75 +721,22 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     CKC(cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming), "event create");
   }
   CKC(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming), "event create");
-  // ligand: centred on the fp32-rounded fp64 centroid (R11); slots in K_SLOTS groups
+  // ligand: centred on the fp32-rounded fp64 centroid (R11)
   float cen[3];
   for (int a = 0; a < 3; ++a) {
     double s = 0.0;
     for (int i = 0; i < n_lig; ++i) s += lig_xyz[3 * i + a];
     cen[a] = (float)(s / n_lig);
   }
-  // slot layout: each group of K_SLOTS = K_PAIRS float2 slot pairs holds its
-  // H-bond-capable atoms (donors / acceptors) in its last pairs; H-bond pairs are spread evenly
-  // over the groups so that the warps of a CTA carry equal work.  Padding slots are all-zero dummy
-  // atoms (exactly zero energy).
-  std::vector<int> plain, hbat;
-  for (int i = 0; i < n_lig; ++i) (don[lig_type[i]] != 0.0f || acc[lig_type[i]] != 0.0f ? hbat : plain).push_back(i);
-  const int pairs_plain = ((int)plain.size() + 1) / 2, pairs_hb = ((int)hbat.size() + 1) / 2;
-  const int groups = (pairs_plain + pairs_hb + K_PAIRS - 1) / K_PAIRS;
-  c->n_chunks = (groups + GROUPS_PER_CTA - 1) / GROUPS_PER_CTA;
-  c->n_groups = c->n_chunks > 1 ? c->n_chunks * GROUPS_PER_CTA : groups;
-  c->hb_base = pairs_hb / c->n_groups;
-  c->hb_extra = pairs_hb % c->n_groups;
-  std::vector<LigSlot> slots((size_t)c->n_groups * K_SLOTS);
-  std::memset(slots.data(), 0, sizeof(LigSlot) * slots.size());
+  // radius of the centred ligand (list reach, R10; item sort grid)
   double rmax = 0.0;
-  std::vector<int> slot_count(c->n_groups, 0);
-  auto put = [&](int slot, int i) {
-    slot_count[slot / K_SLOTS]++;
-    const int t = lig_type[i];
-    LigSlot& s = slots[slot];
-    s.lq.x = lig_xyz[3 * i] - cen[0];
-    s.lq.y = lig_xyz[3 * i + 1] - cen[1];
-    s.lq.z = lig_xyz[3 * i + 2] - cen[2];
-    const double qk = sp.dielectric == 0 ? (double)sp.coulomb_k * lig_q[i] / 4.0
-                                         : (double)sp.coulomb_k * lig_q[i] / (double)sp.eps_r;
-    s.lq.w = (float)qk;
-    s.p = make_float4(c12[t], c6[t], don[t], acc[t]);
-    rmax = std::max(rmax, std::sqrt((double)s.lq.x * s.lq.x + (double)s.lq.y * s.lq.y + (double)s.lq.z * s.lq.z));
-  };
-  {
-    size_t ip = 0, ih = 0;
-    for (int g = 0; g < c->n_groups; ++g) {
-      const int h = c->hb_base + (g < c->hb_extra ? 1 : 0);
-      for (int p = 0; p < K_PAIRS; ++p)
-        for (int half = 0; half < 2; ++half) {
-          const int slot = (g * K_PAIRS + p) * 2 + half;
-          if (p < K_PAIRS - h) {
-            if (ip < plain.size()) put(slot, plain[ip++]);
-          } else if (ih < hbat.size()) {
-            put(slot, hbat[ih++]);
-          }
-        }
-    }
-    if (ip != plain.size() || ih != hbat.size()) {
-      vs_destroy(c);
-      return set_err(VS_ERR_INVALID_ARGUMENT, "internal: ligand slot layout");
-    }
+  for (int i = 0; i < n_lig; ++i) {
+    const double x = (float)(lig_xyz[3 * i] - cen[0]), y = (float)(lig_xyz[3 * i + 1] - cen[1]),
+                 z = (float)(lig_xyz[3 * i + 2] - cen[2]);
+    rmax = std::max(rmax, std::sqrt(x * x + y * y + z * z));
   }
   {
-    // real atoms per group, counted from the placement (an all-zero real atom, e.g. type X at the
-    // centroid, is still counted)
-    std::vector<int> gn(c->n_groups, 0);
-    for (int g = 0; g < c->n_groups; ++g) gn[g] = slot_count[g];
-    CKC(cudaMalloc(&c->d_group_natoms, sizeof(int) * c->n_groups), "alloc");
-    CKC(cudaMemcpy(c->d_group_natoms, gn.data(), sizeof(int) * c->n_groups, cudaMemcpyHostToDevice), "H2D");
-  }
-  CKC(cudaMalloc(&c->d_lig, sizeof(LigSlot) * slots.size()), "alloc ligand");
-  CKC(cudaMemcpy(c->d_lig, slots.data(), sizeof(LigSlot) * slots.size(), cudaMemcpyHostToDevice), "H2D ligand");
-  {
-    // cells engine: ligand atoms in input order; class 1 = H-bond role (donor / acceptor, R5)
-    const char* ev = std::getenv("VS_ENGINE");
-    c->engine = (ev && std::strcmp(ev, "poses") == 0) ? ENGINE_POSES : ENGINE_CELLS;
+    // ligand atoms in input order; class 1 = H-bond role (donor / acceptor, R5)
     std::vector<float4> lx(n_lig), lp(n_lig);
     std::vector<int> rank(n_lig);
     int cnt[2] = {0, 0};
@@ -1075,23 +847,16 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
     CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, (float)(reach * reach), c->d_list_off, nullptr,
                            c->d_lists, 0, c->stream), "list fill launch");
-    // poses engine: distance-sorted lists + shell table (per-warp truncation in the scoring kernel);
-    // cells engine: cell-sorted lists + cell start table (per-chunk culling)
+    // cell-sorted lists + cell start table (per-chunk culling in the pair kernel)
     CKT(cudaMemcpyAsync(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
     RecAtom* sorted = nullptr;
     CKT(cudaMalloc(&sorted, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
-    cudaError_t es;
-    if (c->engine == ENGINE_CELLS) {
-      c->cR = (float)reach + 0.01f;
-      c->ch = 2.0f * c->cR / (float)CELL_G;
-      c->cinv_h = (float)CELL_G / (2.0f * c->cR);
-      CKT(cudaMalloc(&c->d_cells, sizeof(int) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
-      es = launch_cell_sort(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_cells, c->cR, c->cinv_h,
-                            c->stream);
-    } else {
-      CKT(cudaMalloc(&c->d_shell, sizeof(int) * (size_t)n_spots * NSHELL), "alloc shells");
-      es = launch_sort_lists(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_shell, c->stream);
-    }
+    c->cR = (float)reach + 0.01f;
+    c->ch = 2.0f * c->cR / (float)CELL_G;
+    c->cinv_h = (float)CELL_G / (2.0f * c->cR);
+    CKT(cudaMalloc(&c->d_cells, sizeof(int) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
+    cudaError_t es = launch_cell_sort(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_cells, c->cR,
+                                      c->cinv_h, c->stream);
     if (es == cudaSuccess) es = cudaStreamSynchronize(c->stream);
     cudaFree(c->d_lists);
     c->d_lists = sorted;
@@ -1106,13 +871,13 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   CKT(cudaMemcpy(c->d_shift, h_shift.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
   CKT(cudaMalloc(&c->d_iota, sizeof(int) * n_spots), "alloc");
   CKT(cudaMemcpy(c->d_iota, iota.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
-  CKT(cudaMalloc(&c->d_counters, sizeof(unsigned long long) * 2), "alloc");
+  CKT(cudaMalloc(&c->d_counters, sizeof(unsigned long long) * 3), "alloc");
   CKT(cudaMalloc(&c->d_seed, sizeof(uint64_t)), "alloc");
   {
     const char* gv = std::getenv("VS_GRAPHS");
     c->graphs = !(gv && gv[0] == '0');
   }
-  CKT(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 2), "memset");
+  CKT(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 3), "memset");
   CKT(cudaStreamSynchronize(c->stream), "sync");
   free_tmp();
   c->h_list_len = h_len;
@@ -1215,8 +980,8 @@ void vs_destroy(vs_ctx* c) {
   for (auto& b : c->buf) b.release();
   for (auto e : c->ev) cudaEventDestroy(e);
   if (c->gexec) cudaGraphExecDestroy(c->gexec);
-  void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_lig, c->d_iota, c->d_counters,
-                  c->d_seed, c->d_shell, c->d_group_natoms, c->d_cells, c->d_ligx, c->d_ligp, c->d_lig_rank};
+  void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_iota, c->d_counters,
+                  c->d_seed, c->d_cells, c->d_ligx, c->d_ligp, c->d_lig_rank};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   if (c->stream) cudaStreamDestroy(c->stream);
@@ -1244,12 +1009,13 @@ vs_status vs_get_stats(vs_ctx* c, vs_stats* o) {
   CK(cudaDeviceSynchronize(), "sync");
   vs_status s = collect_timing(c);
   if (s != VS_OK) return s;
-  unsigned long long h[2];
+  unsigned long long h[3];
   CK(cudaMemcpy(h, c->d_counters, sizeof(h), cudaMemcpyDeviceToHost), "D2H counters");
   o->kernel_launches = c->launches;
   o->score_launches = c->score_launches;
-  o->pairs = h[0];
+  o->pairs = h[2];
   o->poses_scored = h[1];
+  o->pairs_evaluated = h[0];
   o->score_ms = c->score_ms_acc;
   o->timed_launches = c->timed_acc;
   return VS_OK;
@@ -1260,7 +1026,7 @@ vs_status vs_reset_stats(vs_ctx* c) {
   if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
   DeviceGuard guard(c->dev);
   CK(cudaDeviceSynchronize(), "sync");
-  CK(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 2), "memset");
+  CK(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 3), "memset");
   c->ev_used = 0;
   c->launches = c->score_launches = 0;
   c->score_ms_acc = 0.0;

@@ -2,9 +2,9 @@
 //
 // Philox4x32-10 streams (R23), the fp32 pose operators of the
 // metaheuristic written as single IEEE ops (R24: __f*_rn intrinsics are
-// never contracted into FMA), and the mbarrier / TMA bulk-copy primitives
-// used to stage receptor tiles in shared memory ("tiling via
-// shared memory").  Independent of oracle/ (shares no code with it).
+// never contracted into FMA), and the cp.async primitives used to stage
+// receptor atoms in shared memory ("tiling via shared
+// memory").  Independent of oracle/ (shares no code with it).
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -12,17 +12,11 @@
 namespace vsk {
 
 // ---------------------------------------------------------------- records
-// Receptor atom as streamed by the scoring kernel: 32 B, two float4 so one
+// Receptor atom as streamed by the pair kernel: 32 B, two float4 so one
 // warp-uniform LDS.128 pair broadcasts it to every lane.
 struct __align__(16) RecAtom {
   float4 xq;  // x, y, z relative to the list origin (A), charge q_j (e)
   float4 p;   // c12_j, c6_j, donor_j (0/1), acceptor_j (0/1)
-};
-
-// Ligand slot (K slots per thread-group; padding slots are all-zero).
-struct __align__(16) LigSlot {
-  float4 lq;  // local x, y, z (A), es_i = k q_i / 4 (DDD) or k q_i / eps_r
-  float4 p;   // c12_i, c6_i, donor_i, acceptor_i
 };
 
 // Individual of a population: 32 B.
@@ -99,39 +93,8 @@ __device__ __forceinline__ void perturb(float4& q, float4& t, float dt, float dr
   q = normalize_q(hamilton(dq, q));
 }
 
-// ---------------------------------------------------------------- mbarrier + bulk copy (TMA engine)
+// ---------------------------------------------------------------- asynchronous copies
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
-__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@P1 bra DONE_%=;\n"
-      "bra WAIT_%=;\n"
-      "DONE_%=:\n"
-      "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-
-// 1-D bulk copy global -> shared, completion counted on `bar` (bytes % 16 == 0)
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
 
 // per-thread asynchronous 16-byte copy global -> shared (L2 only), grouped by commit / wait
 __device__ __forceinline__ void cp_async16(void* dst, const void* src) {

@@ -72,9 +72,8 @@ __device__ __forceinline__ uint64_t pkey(float score, uint32_t idx) {
   return ((uint64_t)ord_f32(score) << 32) | idx;
 }
 
-// One CTA per spot.  mode 0: J = best m of S by (score, index) (listed by |t|);
-// mode 1: S_out = S sorted; mode 2: S_out = best P of S ++ C (S first on ties);
-// mode 3: J = the P indices of S ordered by |t| (scoring order).
+// One CTA per spot.  mode 0: J = best m of S by (score, index);
+// mode 1: S_out = S sorted; mode 2: S_out = best P of S ++ C (S first on ties).
 __global__ void popsort_kernel(int mode, const PoseRec* __restrict__ S, const PoseRec* __restrict__ C,
                                PoseRec* __restrict__ S_out, int* __restrict__ J, int P, int m, int N) {
   extern __shared__ uint64_t keys[];
@@ -104,39 +103,8 @@ __global__ void popsort_kernel(int mode, const PoseRec* __restrict__ S, const Po
       __syncthreads();
     }
   }
-  if (mode == 0 || mode == 3) {
-    // mode 0: the best m by (score, index), then re-ordered by distance from the spot centre so that the
-    // scoring warps hold poses of similar |t| (tighter shell truncation; the Improve steps of distinct
-    // elements are independent, so their order does not change any result).
-    // mode 3: all P indices ordered by |t| (scoring order of a population; no result depends on it).
-    const int cnt = mode == 0 ? m : P;
-    __syncthreads();
-    for (int i = threadIdx.x; i < N; i += blockDim.x) {
-      uint64_t key = ~0ull;
-      if (i < cnt) {
-        const uint32_t o = (uint32_t)keys[i];
-        const float4 t = Sk[o].t;
-        key = ((uint64_t)__float_as_uint(t.x * t.x + t.y * t.y + t.z * t.z) << 32) | o;
-      }
-      keys[i] = key;  // same slot read and written by this thread only
-    }
-    __syncthreads();
-    for (int size = 2; size <= N; size <<= 1) {
-      for (int stride = size >> 1; stride > 0; stride >>= 1) {
-        for (int i = threadIdx.x; i < (N >> 1); i += blockDim.x) {
-          const int lo = 2 * i - (i & (stride - 1));
-          const int hi = lo + stride;
-          const bool asc = (lo & size) == 0;
-          const uint64_t a = keys[lo], b = keys[hi];
-          if ((a > b) == asc) {
-            keys[lo] = b;
-            keys[hi] = a;
-          }
-        }
-        __syncthreads();
-      }
-    }
-    for (int r = threadIdx.x; r < cnt; r += blockDim.x) J[(size_t)k * cnt + r] = (int)(uint32_t)keys[r];
+  if (mode == 0) {  // the best m by (score, index), in that order
+    for (int r = threadIdx.x; r < m; r += blockDim.x) J[(size_t)k * m + r] = (int)(uint32_t)keys[r];
   } else {
     for (int r = threadIdx.x; r < P; r += blockDim.x) {
       const int o = (int)(uint32_t)keys[r];
@@ -201,58 +169,6 @@ __global__ void list_kernel(const float4* __restrict__ rec, const float4* __rest
   if (threadIdx.x == 0 && count_only) len[s] = base_sh;
 }
 
-// One CTA per spot: (|r|^2, index) keys bitonic-sorted in shared memory, records gathered into tmp
-// in distance order (ties by list position: deterministic), shell prefix counts by binary search.
-// Lists longer than SORT_MAX stay unsorted and get a flat shell table (no truncation).
-__global__ void sort_lists_kernel(const RecAtom* __restrict__ lists, RecAtom* __restrict__ tmp, const int* off,
-                                  const int* len, int* shell) {
-  extern __shared__ uint64_t skeys[];
-  const int s = blockIdx.x;
-  const int n = len[s];
-  const RecAtom* L = lists + off[s];
-  RecAtom* O = tmp + off[s];
-  int* sh = shell + (size_t)s * NSHELL;
-  if (n > SORT_MAX) {
-    for (int i = threadIdx.x; i < n; i += blockDim.x) O[i] = L[i];
-    for (int b = threadIdx.x; b < NSHELL; b += blockDim.x) sh[b] = n;
-    return;
-  }
-  int N = 1;
-  while (N < n) N <<= 1;
-  for (int i = threadIdx.x; i < N; i += blockDim.x) {
-    uint64_t key = ~0ull;
-    if (i < n) {
-      const float4 x = L[i].xq;
-      const float d2 = x.x * x.x + x.y * x.y + x.z * x.z;
-      key = ((uint64_t)__float_as_uint(d2) << 32) | (uint32_t)i;
-    }
-    skeys[i] = key;
-  }
-  __syncthreads();
-  for (int size = 2; size <= N; size <<= 1)
-    for (int stride = size >> 1; stride > 0; stride >>= 1) {
-      for (int i = threadIdx.x; i < (N >> 1); i += blockDim.x) {
-        const int lo = 2 * i - (i & (stride - 1)), hi = lo + stride;
-        const bool asc = (lo & size) == 0;
-        const uint64_t a = skeys[lo], b = skeys[hi];
-        if ((a > b) == asc) { skeys[lo] = b; skeys[hi] = a; }
-      }
-      __syncthreads();
-    }
-  for (int i = threadIdx.x; i < n; i += blockDim.x) O[i] = L[(uint32_t)skeys[i]];
-  // shell[b] = #atoms with |r|^2 < ((b+1) DR)^2  (upper bound search on the sorted d^2)
-  for (int b = threadIdx.x; b < NSHELL; b += blockDim.x) {
-    const float R = (float)(b + 1) * SHELL_DR;
-    const uint32_t lim = __float_as_uint(R * R);
-    int lo = 0, hi = n;
-    while (lo < hi) {
-      const int mid = (lo + hi) >> 1;
-      if ((uint32_t)(skeys[mid] >> 32) < lim) lo = mid + 1; else hi = mid;
-    }
-    sh[b] = lo;
-  }
-}
-
 __global__ void philox_kernel(int64_t n, const uint4* ctr, uint2 key, uint4* out) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) out[i] = philox4x32_10(ctr[i], key);
@@ -277,40 +193,6 @@ __global__ void validate_kernel(int64_t n, const int32_t* spot, const float* q, 
   valid[i] = ok ? 1 : 0;
   if (ok) atomicAdd(counts + s, 1);
   else score_out[i] = __int_as_float(0x7fc00000);
-}
-
-// exclusive prefix of per-spot counts -> pose_prefix, blk_prefix (+cursor copy); one CTA
-__global__ void scan_kernel(const int* counts, int n, int* pose_prefix, int* blk_prefix, int* cursor) {
-  __shared__ int part[1024];
-  __shared__ int bpart[1024];
-  __shared__ int carry, bcarry;
-  if (threadIdx.x == 0) { carry = 0; bcarry = 0; }
-  __syncthreads();
-  for (int b = 0; b < n; b += blockDim.x) {
-    const int i = b + threadIdx.x;
-    const int c = i < n ? counts[i] : 0;
-    const int bc = (c + POSES_PER_CTA - 1) / POSES_PER_CTA;
-    part[threadIdx.x] = c;
-    bpart[threadIdx.x] = bc;
-    __syncthreads();
-    for (int o = 1; o < (int)blockDim.x; o <<= 1) {  // Hillis-Steele inclusive scan
-      int v = threadIdx.x >= (unsigned)o ? part[threadIdx.x - o] : 0;
-      int bv = threadIdx.x >= (unsigned)o ? bpart[threadIdx.x - o] : 0;
-      __syncthreads();
-      part[threadIdx.x] += v;
-      bpart[threadIdx.x] += bv;
-      __syncthreads();
-    }
-    if (i < n) {
-      pose_prefix[i] = carry + part[threadIdx.x] - c;
-      blk_prefix[i] = bcarry + bpart[threadIdx.x] - bc;
-      cursor[i] = pose_prefix[i];
-    }
-    __syncthreads();
-    if (threadIdx.x == blockDim.x - 1) { carry += part[threadIdx.x]; bcarry += bpart[threadIdx.x]; }
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) { pose_prefix[n] = carry; blk_prefix[n] = bcarry; }
 }
 
 __global__ void scatter_kernel(int64_t n, const int32_t* spot, const float* q, const float* t, const int* valid,
@@ -363,12 +245,6 @@ cudaError_t launch_build_lists(const float4* rec, const float4* rprm, int n_rec,
   return cudaGetLastError();
 }
 
-cudaError_t launch_sort_lists(RecAtom* lists, RecAtom* tmp, const int* off, const int* len, int n_spots, int* shell,
-                              cudaStream_t st) {
-  sort_lists_kernel<<<n_spots, 1024, sizeof(uint64_t) * SORT_MAX, st>>>(lists, tmp, off, len, shell);
-  return cudaGetLastError();
-}
-
 cudaError_t launch_philox(int64_t n, const uint4* ctr, uint2 key, uint4* out, cudaStream_t st) {
   if (n <= 0) return cudaSuccess;
   philox_kernel<<<nblk(n, 256), 256, 0, st>>>(n, ctr, key, out);
@@ -378,11 +254,6 @@ cudaError_t launch_philox(int64_t n, const uint4* ctr, uint2 key, uint4* out, cu
 cudaError_t launch_validate(int64_t n, const int32_t* spot, const float* q, const float* t, int n_spots, float T,
                             int cutoff, int* valid, int* counts, float* score_out, cudaStream_t st) {
   validate_kernel<<<nblk(n, 256), 256, 0, st>>>(n, spot, q, t, n_spots, T, cutoff, valid, counts, score_out);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_scan(const int* counts, int n, int* pose_prefix, int* blk_prefix, int* cursor, cudaStream_t st) {
-  scan_kernel<<<1, 1024, 0, st>>>(counts, n, pose_prefix, blk_prefix, cursor);
   return cudaGetLastError();
 }
 

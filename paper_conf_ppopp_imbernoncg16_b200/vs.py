@@ -46,7 +46,8 @@ class MHParams(C.Structure):
 
 class Stats(C.Structure):
     _fields_ = [("kernel_launches", C.c_uint64), ("score_launches", C.c_uint64), ("poses_scored", C.c_uint64),
-                ("pairs", C.c_uint64), ("score_ms", C.c_double), ("timed_launches", C.c_uint64)]
+                ("pairs", C.c_uint64), ("score_ms", C.c_double), ("timed_launches", C.c_uint64),
+                ("pairs_evaluated", C.c_uint64)]
 
     def asdict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -213,9 +213,10 @@ def test_device_entry_point(gpu, oracle_mod):
 
 
 def test_stats_count_pairs(gpu, oracle_mod):
-    """Pairs counted = real ligand atoms x receptor atoms streamed.  All-pairs mode streams the whole receptor;
-    cutoff mode streams a subset of each spot's list (cells engine: the cell rows within rc of each chunk's
-    bounding box; poses engine: each warp's inner shells of the distance-sorted list)."""
+    """`pairs` = workload pairs, n_lig x list length of the pose's spot per scored pose (the whole receptor in
+    all-pairs mode); `pairs_evaluated` = item slots x receptor atoms streamed per chunk: every list atom in
+    all-pairs mode (plus the padding slots of a chunk), in cutoff mode only the cell rows within rc of a
+    chunk's bounding box."""
     prob = synth.make_problem("tiny")
     spot, q, t = synth.make_poses(100, 4, 3.0, seed=2)
     g, _ = both(oracle_mod, prob, 0.0)
@@ -223,7 +224,9 @@ def test_stats_count_pairs(gpu, oracle_mod):
     g.set_timing(True)
     g.score_poses(spot, q, t)
     st = g.stats()
-    assert st["poses_scored"] == 100 and st["pairs"] == 100 * prob.cfg.n_rec * prob.cfg.n_lig
+    full = 100 * prob.cfg.n_rec * prob.cfg.n_lig
+    assert st["poses_scored"] == 100 and st["pairs"] == full
+    assert full <= st["pairs_evaluated"] <= 1.5 * full
     assert st["score_launches"] == 1 and st["timed_launches"] == 1 and st["score_ms"] > 0
     gm = vs.Context.from_problem(synth.make_problem("medium"), vs.score_params(cutoff=12.0))
     pm = synth.make_problem("medium")
@@ -232,26 +235,10 @@ def test_stats_count_pairs(gpu, oracle_mod):
     gm.score_poses(spot, q, t)
     st = gm.stats()
     full = int(sum(int(gm.list_lengths()[s]) for s in spot)) * pm.cfg.n_lig
-    assert st["poses_scored"] == 4000 and 0.25 * full < st["pairs"] < full     # culling skips 30-55 %
-
-
-def test_scores_independent_of_batch_composition(gpu, oracle_mod):
-    """A pose's score depends only on the pose and its spot: scoring it alone, inside a larger batch, or in a
-    shuffled batch gives the same bits (the cells engine sorts each spot's atoms spatially and culls per
-    chunk; out-of-cutoff pairs add exactly zero and in-cutoff pairs are summed in list order)."""
-    prob = synth.make_problem("small")
-    g, o = both(oracle_mod, prob, 12.0)
-    spot, q, t = synth.make_poses(3000, prob.cfg.n_spots, 3.0, seed=11)
-    full = g.score_poses(spot, q, t)
-    perm = np.random.default_rng(3).permutation(3000)
-    shuf = np.empty_like(full)
-    shuf[perm] = g.score_poses(spot[perm], q[perm], t[perm])
-    np.testing.assert_array_equal(full, shuf)
-    sub = np.arange(0, 3000, 7)
-    np.testing.assert_array_equal(full[sub], g.score_poses(spot[sub], q[sub], t[sub]))
-    for i in (0, 1234, 2999):
-        np.testing.assert_array_equal(full[i:i + 1], g.score_poses(spot[i:i + 1], q[i:i + 1], t[i:i + 1]))
-    assert_scores(full[::60], o.score(spot[::60], q[::60], t[::60]))
+    assert st["poses_scored"] == 4000 and st["pairs"] == full
+    assert 0.25 * full < st["pairs_evaluated"] < full     # culling skips 30-60 %
+    sc = gm.score_poses(spot[:1], q[:1], t[:1])
+    assert gm.stats()["pairs"] == full + int(gm.list_lengths()[spot[0]]) * pm.cfg.n_lig and np.isfinite(sc).all()
 
 
 # ------------------------------------------------------------------ metaheuristic
@@ -352,12 +339,12 @@ def test_lockstep_trace(gpu, oracle_mod, preset, P, G, K):
                 assert_scores(pop[s, :, 7], o.score(np.full(P, s, np.int32), pop[s, :, :4], pop[s, :, 4:7]))
             prev = pop
         elif stage == vs.TRACE_SELECT:
-            # the selected set is exact; the GPU lists it by |t| (scoring order only)
+            # the selected set is exact, listed in (score, index) order
             for s in spots:
                 want = oracle_mod.select_improve(prev[s, :, 7].astype(np.float64), m)
                 np.testing.assert_array_equal(np.sort(idx[s]), np.sort(want))
-                tn = (prev[s, idx[s], 4:7].astype(np.float32) ** 2).sum(1)
-                assert np.all(np.diff(tn) >= -1e-6)
+                sc = prev[s, idx[s], 7]
+                assert np.all((np.diff(sc) > 0) | ((np.diff(sc) == 0) & (np.diff(idx[s]) > 0)))
             J = idx
         elif stage == vs.TRACE_LS:
             for s in spots:
