@@ -16,7 +16,7 @@ def shares(path):
         if len(r) <= vi:
             continue
         name = r[ki] if "cell_pair" in r[ki] or "score_kernel" in r[ki] else r[ki].split("(")[0]
-        v = float(r[vi].replace(",", "")) * {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3}.get(r[ui], 1.0)
+        v = float(r[vi].replace(",", "")) * {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "msecond": 1e3}.get(r[ui], 1.0)
         agg[name][0] += 1
         agg[name][1] += v
     tot = sum(v[1] for v in agg.values())
