@@ -115,6 +115,40 @@ def test_ragged_ligand_sizes(gpu, oracle_mod, n_lig):
         assert_scores(g.score_poses(spot, q, t), o.score(spot, q, t), f"n_lig={n_lig} rc={cutoff}")
 
 
+@pytest.mark.parametrize("mix", ["no_hbond", "all_hbond", "hbond_heavy"])
+def test_ligand_class_mixes(gpu, oracle_mod, mix):
+    """Ligands whose H-bond-capable share selects every slot layout: none (H = 0), only H-bond atoms
+    (H = CELL_KP, no class-0 slots) and more H-bond than other atoms (class-0 items overflowing or not);
+    ragged pose counts per spot give partially filled chunks; scoring and a short M3 / N4 run."""
+    prob = synth.make_custom(2500, 23, 6, seed=17)
+    rng = np.random.default_rng(5)
+    pick = {"no_hbond": [synth.T_C, synth.T_H, synth.T_S], "all_hbond": [synth.T_N, synth.T_O, synth.T_HD],
+            "hbond_heavy": [synth.T_N, synth.T_O, synth.T_HD, synth.T_HD, synth.T_C]}[mix]
+    prob.lig.type[:] = rng.choice(pick, size=len(prob.lig.type)).astype(np.int32)
+    for cutoff in (12.0, 0.0):
+        g, o = both(oracle_mod, prob, cutoff)
+        spot, q, t = synth.make_poses(301, 6, 3.0, seed=9)
+        spot[:37] = 2                                       # one crowded spot, others ragged
+        assert_scores(g.score_poses(spot, q, t), o.score(spot, q, t), f"{mix} rc={cutoff}")
+    g, o = both(oracle_mod, prob, 12.0)
+    for K in (1, 3):
+        _, sg = g.run(vs.mh_preset(3, population=24, generations=2, ls_neighbours=K), 8)
+        _, so = o.run(oracle_mod.mh_preset(3, population=24, generations=2, ls_neighbours=K), 8)
+        assert np.all(np.abs(sg - so) <= 1e-3 * np.maximum(np.abs(so), 1.0)), (mix, K, sg, so)
+
+
+def test_long_lists_streamed_whole(gpu, oracle_mod):
+    """Cutoff lists longer than the cell sort's limit (16384 atoms: here rc = 70 A on a 25k-atom receptor)
+    are streamed whole instead of cell-culled; scores still match the brute-force cutoff definition."""
+    prob = synth.make_custom(25000, 30, 3, seed=23)
+    g, o = both(oracle_mod, prob, 70.0)
+    assert g.list_lengths().max() > 16384
+    spot, q, t = synth.make_poses(200, 3, 3.0, seed=4)
+    got = g.score_poses(spot, q, t)
+    idx = np.arange(0, 200, 25)
+    assert_scores(got[idx], o.score(spot[idx], q[idx], t[idx]))
+
+
 def test_list_tiles_ragged_and_empty(gpu, oracle_mod):
     """Spot far outside the receptor (empty cutoff list) and list lengths across tile boundaries."""
     prob = synth.make_custom(700, 13, 4, seed=2)
