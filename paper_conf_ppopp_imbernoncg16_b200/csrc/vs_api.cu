@@ -104,7 +104,7 @@ struct vs_ctx {
   int* d_iota = nullptr;
   unsigned long long* d_counters = nullptr;  // [0] pairs evaluated, [1] poses, [2] workload pairs
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
-  int* d_cells = nullptr;               // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
+  uint16_t* d_cells = nullptr;          // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
   float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
   float4* d_ligx = nullptr;             // [n_lig] centred local coordinates, w = class
   float4* d_ligp = nullptr;             // [n_lig] es, c12, c6, donor
@@ -854,7 +854,7 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     c->cR = (float)reach + 0.01f;
     c->ch = 2.0f * c->cR / (float)CELL_G;
     c->cinv_h = (float)CELL_G / (2.0f * c->cR);
-    CKT(cudaMalloc(&c->d_cells, sizeof(int) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
+    CKT(cudaMalloc(&c->d_cells, sizeof(uint16_t) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
     cudaError_t es = launch_cell_sort(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_cells, c->cR,
                                       c->cinv_h, c->stream);
     if (es == cudaSuccess) es = cudaStreamSynchronize(c->stream);

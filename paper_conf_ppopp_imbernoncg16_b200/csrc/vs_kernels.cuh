@@ -13,7 +13,13 @@ enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
 // Work unit = chunk of up to CH_ITEMS transformed ligand atoms ("items": one ligand atom of one pose),
 // spatially sorted per spot; the chunk streams only the cell rows of the spot's cell-sorted list
 // within rc of its bounding box.
-constexpr int CELL_G = 24;                         // list grid per spot: G^3 cells over [-R, R]^3
+#ifndef VS_CELL_G
+#define VS_CELL_G 32
+#endif
+#ifndef VS_CELL_EXACTX
+#define VS_CELL_EXACTX 1
+#endif
+constexpr int CELL_G = VS_CELL_G;                  // list grid per spot: G^3 cells over [-R, R]^3 (G <= 64)
 constexpr int CELL_G3 = CELL_G * CELL_G * CELL_G;
 constexpr int CELL_SORT_MAX = 16384;               // longest list cell-sorted in shared memory (128 KB keys)
 #ifndef VS_CELL_KP
@@ -30,12 +36,12 @@ constexpr int MORTON_BITS = 4;                     // item sort grid: 16^3 cells
 constexpr int MORTON_BINS = 1 << (3 * MORTON_BITS);
 
 struct CellArgs {
-  // receptor lists (per spot) and the cell start table [n_spots][CELL_G3 + 1] (list positions;
-  // cells[s][0] < 0: list not cell-sorted -> streamed whole)
+  // receptor lists (per spot) and the cell start table [n_spots][CELL_G3 + 1] (uint16 list positions; a
+  // cell-sorted list has <= CELL_SORT_MAX < 2^16 atoms; cells[s][0] == 0xFFFF: not cell-sorted -> streamed whole)
   const RecAtom* lists;
   const int* list_off;
   const int* list_len;
-  const int* cells;
+  const uint16_t* cells;
   float cR, ch, cinv_h;      // grid half-width (A), cell edge, 1 / edge
   // ligand (input order)
   const float4* ligx;        // local x, y, z (centred), w = class (0: no H-bond role, 1: donor / acceptor)
@@ -89,7 +95,7 @@ __host__ __device__ inline int cell_chunks(int seg_n, int nn, int nh, int cap, i
   return (int)c;
 }
 
-cudaError_t launch_cell_sort(const RecAtom* lists, RecAtom* out, const int* off, const int* len, int n_spots, int* cells,
+cudaError_t launch_cell_sort(const RecAtom* lists, RecAtom* out, const int* off, const int* len, int n_spots, uint16_t* cells,
                              float R, float inv_h, cudaStream_t st);
 // K1 + K2 + K3 of one scoring call; n_blocks2 = pair-kernel grid (upper bound when non-uniform)
 cudaError_t launch_cell_score(const CellArgs& a, int dielectric, long long n_poses, int n_blocks2, cudaStream_t st);
