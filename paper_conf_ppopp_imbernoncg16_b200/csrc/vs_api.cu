@@ -69,7 +69,10 @@ struct DevBuf {
 #define VS_NSUB 4
 #endif
 constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
-constexpr int MAX_SPLIT = 8;  // receptor-list splits of one scoring launch (cell_nsplit)
+#ifndef VS_MAX_SPLIT
+#define VS_MAX_SPLIT 8
+#endif
+constexpr int MAX_SPLIT = VS_MAX_SPLIT;  // receptor-list splits of one scoring launch (cell_nsplit; a power of 2)
 #ifndef VS_GROUP_SPOTS
 #define VS_GROUP_SPOTS 16   // spots per stream group at least
 #endif
