@@ -73,11 +73,18 @@ constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
 #define VS_MAX_SPLIT 8
 #endif
 constexpr int MAX_SPLIT = VS_MAX_SPLIT;  // receptor-list splits of one scoring launch (cell_nsplit; a power of 2)
+static_assert(vsk::CELL_G % MAX_SPLIT == 0, "the pair kernel assigns cell rows to splits by cy mod nsplit");
 #ifndef VS_GROUP_SPOTS
 #define VS_GROUP_SPOTS 16   // spots per stream group at least
 #endif
 #ifndef VS_SPLIT_WARPS
-#define VS_SPLIT_WARPS 16
+#define VS_SPLIT_WARPS 16     // chunks x splits per spot at least ...
+#endif
+#ifndef VS_SPLIT_WARPS_MAX
+#define VS_SPLIT_WARPS_MAX 64  // ... raised for contexts with few spots, up to this
+#endif
+#ifndef VS_SPLIT_TOTAL
+#define VS_SPLIT_TOTAL 4096    // pair-kernel warps a launch over all spots of the context should reach (~1 wave)
 #endif
 
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
@@ -109,6 +116,7 @@ struct vs_ctx {
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
   uint16_t* d_cells = nullptr;          // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
   float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
+  int split_warps = VS_SPLIT_WARPS;     // cell_nsplit target, fixed at vs_create from n_spots
   float4* d_ligx = nullptr;             // [n_lig] centred local coordinates, w = class
   float4* d_ligp = nullptr;             // [n_lig] es, c12, c6, donor
   int* d_lig_rank = nullptr;            // [n_lig] rank within the class
@@ -186,11 +194,13 @@ vs_status collect_timing(vs_ctx* c) {
   return VS_OK;
 }
 
-// list splits of a scoring launch: chunks per spot below VS_SPLIT_WARPS are split over up to MAX_SPLIT
-// list ranges.  Depends only on per-spot quantities (bitwise independence of the spot chunking / GPU count).
-int cell_nsplit(int nch) {
+// list splits of a scoring launch: a spot whose chunks number fewer than split_warps has its cell rows dealt
+// over up to MAX_SPLIT splits.  split_warps is a property of the context (set at vs_create from n_spots: few
+// spots, small launches, more splits), so the choice depends on per-spot quantities and the context only --
+// results stay bitwise identical across spot chunkings of a run and GPU counts.
+int cell_nsplit(int nch, int split_warps) {
   int ns = 1;
-  while (ns < MAX_SPLIT && (long)nch * ns < VS_SPLIT_WARPS) ns *= 2;
+  while (ns < MAX_SPLIT && (long)nch * ns < split_warps) ns *= 2;
   return ns;
 }
 
@@ -404,7 +414,7 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
       cp.P = P;
       cp.mode = MODE_PLAIN;
       cp.nch_u = cell_chunks(P, c->nn, c->nh, c->cn, c->chb);
-      cp.nsplit = cell_nsplit(cp.nch_u);
+      cp.nsplit = cell_nsplit(cp.nch_u, c->split_warps);
       cp.pbuf = b.pbuf + (size_t)k0 * maxpose;
       cp.items = b.items + (size_t)k0 * maxpose * c->n_lig;
       cp.E = b.E + (size_t)k0 * c->n_lig * b.emax;
@@ -414,7 +424,7 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
       cl.mode = MODE_LS;
       cl.seg_size = mk;
       cl.nch_u = cell_chunks(mk, c->nn, c->nh, c->cn, c->chb);
-      cl.nsplit = cell_nsplit(cl.nch_u);
+      cl.nsplit = cell_nsplit(cl.nch_u, c->split_warps);
       cl.E_stride = (long long)q.ns * mk * c->n_lig;
       cl.J = q.J;
       cl.m = m;
@@ -467,8 +477,8 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     const int mk = m * mp->ls_neighbours, maxpose = std::max(P, mk);
     if ((long long)ns * maxpose * c->n_lig >= (1ll << 31))
       return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel x population x n_lig must be < 2^31");
-    emax = P * cell_nsplit(cell_chunks(P, c->nn, c->nh, c->cn, c->chb));
-    if (mp->improve_frac > 0.0f) emax = std::max(emax, mk * cell_nsplit(cell_chunks(mk, c->nn, c->nh, c->cn, c->chb)));
+    emax = P * cell_nsplit(cell_chunks(P, c->nn, c->nh, c->cn, c->chb), c->split_warps);
+    if (mp->improve_frac > 0.0f) emax = std::max(emax, mk * cell_nsplit(cell_chunks(mk, c->nn, c->nh, c->cn, c->chb), c->split_warps));
     CK(c->buf[B_PBUF].ensure(sizeof(PoseRec) * (size_t)ns * maxpose), "alloc");
     CK(c->buf[B_ITEMS].ensure(sizeof(float4) * (size_t)ns * maxpose * c->n_lig), "alloc");
     CK(c->buf[B_E].ensure(sizeof(double) * (size_t)ns * c->n_lig * emax), "alloc");
@@ -698,6 +708,7 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   c->n_rec = n_rec;
   c->n_lig = n_lig;
   c->n_spots = n_spots;
+  c->split_warps = std::max(VS_SPLIT_WARPS, std::min(VS_SPLIT_WARPS_MAX, VS_SPLIT_TOTAL / std::max(1, (int)n_spots)));
   c->all_pairs = !(sp.cutoff > 0.0f) || std::isinf(sp.cutoff);
   c->dielectric = sp.dielectric;
   c->T = sp.region_half_width;
