@@ -32,6 +32,11 @@ import time
 
 import numpy as np
 
+# One vs_run drives up to 9 streams per context (main + spot groups): give them their own hardware work queues
+# (the default 8 aliases streams onto shared queues; measured: context create / destroy costs become erratic,
+# up to hundreds of ms).  Must be set before the CUDA context exists.
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
@@ -386,7 +391,7 @@ def main():
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
-        parts_ms = {"create": 0.0, "run": 0.0, "destroy": 0.0}
+        parts_ms = {"create": 0.0, "run": 0.0, "stats": 0.0, "destroy": 0.0}
         for i in range(n_e2e):
             # sweep: this rank's share of the ligands (static round robin), one context per ligand
             for li in (range(rank, len(ligs), world) if sweep else [0]):
@@ -396,11 +401,13 @@ def main():
                 c2.run(mp, (screen.ligand_seed(args.seed, li) if sweep else args.seed + rank), None)
                 tc = time.perf_counter()
                 e2e_ctx_stats.append(c2.stats())
+                tcs = time.perf_counter()
                 c2.close()
                 td = time.perf_counter()
                 parts_ms["create"] += 1e3 * (tb - ta)
                 parts_ms["run"] += 1e3 * (tc - tb)
-                parts_ms["destroy"] += 1e3 * (td - tc)
+                parts_ms["stats"] += 1e3 * (tcs - tc)
+                parts_ms["destroy"] += 1e3 * (td - tcs)
         dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=cdev)
         e2e_pairs = torch.tensor([sum(s["pairs"] for s in e2e_ctx_stats)], dtype=torch.float64, device=cdev)
         if world > 1:

@@ -66,7 +66,7 @@ struct DevBuf {
 };
 
 #ifndef VS_NSUB
-#define VS_NSUB 4
+#define VS_NSUB 8
 #endif
 constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
 #ifndef VS_MAX_SPLIT
@@ -75,7 +75,13 @@ constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
 constexpr int MAX_SPLIT = VS_MAX_SPLIT;  // receptor-list splits of one scoring launch (cell_nsplit; a power of 2)
 static_assert(vsk::CELL_G % MAX_SPLIT == 0, "the pair kernel assigns cell rows to splits by cy mod nsplit");
 #ifndef VS_GROUP_SPOTS
-#define VS_GROUP_SPOTS 16   // spots per stream group at least
+#define VS_GROUP_SPOTS 8    // spots per stream group at least
+#endif
+#ifndef VS_BIG_RUN_SPOTS
+#define VS_BIG_RUN_SPOTS 256  // runs of at least this many spots use at most VS_BIG_RUN_GROUPS streams
+#endif
+#ifndef VS_BIG_RUN_GROUPS
+#define VS_BIG_RUN_GROUPS 8
 #endif
 #ifndef VS_SPLIT_WARPS
 #define VS_SPLIT_WARPS 16     // chunks x splits per spot at least ...
@@ -388,7 +394,12 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
   // Spots are independent: split them into groups whose generation loops run on separate
   // streams, enqueued generation by generation, so one group's kernels fill the wave tails of
   // another's.
-  const int G = tr ? 1 : std::max(1, std::min(NSUB, ns / VS_GROUP_SPOTS));
+  // Stream count (measured on B200, profiles/r01_notes.md): small runs are chains of latency-bound launches and
+  // gain from every extra stream (64 spots: 4 -> 16 streams, 25.8 -> 23.1 ms / step); large runs fill the GPU
+  // with 8 (500 spots: 8 streams 598 ms, 16 streams 603 ms).
+  int G = std::max(1, std::min(NSUB, ns / VS_GROUP_SPOTS));
+  if (ns >= VS_BIG_RUN_SPOTS) G = std::min(G, VS_BIG_RUN_GROUPS);
+  if (tr) G = 1;
   Group grp[NSUB];
   CK(cudaEventRecord(c->ev_fork, st), "event record");
   for (int gi = 0; gi < G; ++gi) {

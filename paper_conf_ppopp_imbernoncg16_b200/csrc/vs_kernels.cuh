@@ -7,6 +7,49 @@
 
 namespace vsk {
 
+// ---------------------------------------------------------------- programmatic dependent launch (PDL)
+// The kernels of a run's per-stream chain (init / combine / popsort / best and the three scoring kernels) are
+// launched with programmatic stream serialization, so a kernel may be scheduled while its predecessor drains; its
+// first statement (griddepcontrol.wait) blocks until the predecessor grid has completed and its memory is
+// visible, so only launch latency is overlapped (small config 25.8 -> 24.9 ms / step).  With VS_PDL_TRIGGER the
+// chain kernels also signal launch_dependents at entry; measured on B200 that lets waiting dependents hold SM
+// slots the other spot-group streams need (medium 602 -> 785 ms / step), so it is off.
+#ifndef VS_PDL
+#define VS_PDL 1
+#endif
+#ifndef VS_PDL_TRIGGER
+#define VS_PDL_TRIGGER 0
+#endif
+
+__device__ __forceinline__ void pdl_enter() {
+#if VS_PDL
+  asm volatile("griddepcontrol.wait;\n" ::: "memory");
+#if VS_PDL_TRIGGER
+  asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
+#endif
+#endif
+}
+
+template <typename... KP, typename... AP>
+cudaError_t launch_chain(void (*k)(KP...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, AP... args) {
+#if VS_PDL
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k, args...);
+#else
+  k<<<grid, block, smem, st>>>(args...);
+  return cudaGetLastError();
+#endif
+}
+
 enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
 
 // ---------------------------------------------------------------- scoring (vs_cells.cu)
