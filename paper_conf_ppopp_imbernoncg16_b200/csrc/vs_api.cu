@@ -7,10 +7,13 @@
 // groups on up to 4 streams, captured as one CUDA graph on repeated calls),
 // and the device boundary is crossed at the start (seed, spot ids) and the
 // end (best pose + score per spot).
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
+#include <unordered_map>
 #include <new>
 #include <string>
 #include <vector>
@@ -46,20 +49,130 @@ struct DeviceGuard {
   }
 };
 
+// ---------------------------------------------------------------- device memory cache
+// A context allocates ~20 device buffers at vs_create / first vs_run and frees them at vs_destroy; on the B200 box
+// cudaMalloc / cudaFree cost 1-30 ms each, erratically (measured inside vs_destroy with VS_DEBUG_TIMING), which
+// dominated the end-to-end time of short runs and of the one-context-per-ligand sweep.  Freed blocks are kept per
+// device and handed to later allocations of the same bucket (size rounded up to a power of two below 2 MiB, to a
+// 2 MiB multiple above).  Cached free bytes per device are capped (VS_POOL_CACHE_MB, default 8192); beyond that,
+// and for pointers the cache did not allocate, frees go to the driver.  A block is returned only when no GPU work
+// can still use it: every caller synchronises first (vs_destroy, DevBuf regrow, the end of vs_create).
+namespace pool {
+struct Dev {
+  std::unordered_map<size_t, std::vector<void*>> free;
+  std::unordered_map<void*, size_t> live;
+  size_t cached = 0;
+};
+std::mutex mu;
+std::unordered_map<int, Dev>& devs() {
+  static auto* d = new std::unordered_map<int, Dev>();  // never destroyed: frees may run during process teardown
+  return *d;
+}
+size_t bucket(size_t b) {
+  constexpr size_t big = size_t(2) << 20;
+  if (b <= big) {
+    size_t k = 512;
+    while (k < b) k <<= 1;
+    return k;
+  }
+  return (b + big - 1) / big * big;
+}
+size_t cache_cap() {
+  static const size_t cap = [] {
+    const char* v = std::getenv("VS_POOL_CACHE_MB");
+    return (size_t)(v ? std::strtoull(v, nullptr, 10) : 8192ull) << 20;
+  }();
+  return cap;
+}
+void trim(int dev) {  // hand every cached block of dev back to the driver
+  std::vector<void*> ps;
+  {
+    std::lock_guard<std::mutex> g(mu);
+    Dev& d = devs()[dev];
+    for (auto& kv : d.free)
+      for (void* q : kv.second) ps.push_back(q);
+    d.free.clear();
+    d.cached = 0;
+  }
+  for (void* q : ps) cudaFree(q);
+}
+cudaError_t alloc(void** p, size_t bytes) {
+  *p = nullptr;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const size_t b = bucket(std::max<size_t>(bytes, 1));
+  {
+    std::lock_guard<std::mutex> g(mu);
+    Dev& d = devs()[dev];
+    auto it = d.free.find(b);
+    if (it != d.free.end() && !it->second.empty()) {
+      *p = it->second.back();
+      it->second.pop_back();
+      d.cached -= b;
+      d.live[*p] = b;
+      return cudaSuccess;
+    }
+  }
+  cudaError_t e = cudaMalloc(p, b);
+  if (e == cudaErrorMemoryAllocation) {  // cached blocks of other sizes may be what is missing
+    cudaGetLastError();
+    trim(dev);
+    e = cudaMalloc(p, b);
+  }
+  if (e != cudaSuccess) {
+    *p = nullptr;
+    return e;
+  }
+  std::lock_guard<std::mutex> g(mu);
+  devs()[dev].live[*p] = b;
+  return cudaSuccess;
+}
+template <typename T>
+cudaError_t alloc(T** p, size_t bytes) {
+  void* q = nullptr;
+  const cudaError_t e = alloc(&q, bytes);
+  *p = static_cast<T*>(q);
+  return e;
+}
+void release(void* p) {
+  if (!p) return;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> g(mu);
+    Dev& d = devs()[dev];
+    auto it = d.live.find(p);
+    if (it != d.live.end()) {
+      const size_t b = it->second;
+      d.live.erase(it);
+      if (d.cached + b <= cache_cap()) {
+        d.free[b].push_back(p);
+        d.cached += b;
+        return;
+      }
+    }
+  }
+  cudaFree(p);
+}
+}  // namespace pool
+
 struct DevBuf {
   void* p = nullptr;
   size_t cap = 0;
   cudaError_t ensure(size_t bytes) {
     if (bytes <= cap) return cudaSuccess;
-    if (p) cudaFree(p);
+    if (p) {
+      cudaDeviceSynchronize();  // earlier launches may still read the old block
+      pool::release(p);
+    }
     p = nullptr;
     cap = 0;
-    cudaError_t e = cudaMalloc(&p, bytes);
+    cudaError_t e = pool::alloc(&p, bytes);
     if (e == cudaSuccess) cap = bytes;
     return e;
   }
   void release() {
-    if (p) cudaFree(p);
+    pool::release(p);
     p = nullptr;
     cap = 0;
   }
@@ -791,12 +904,12 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     }
     c->cn = CH_ITEMS;
     c->chb = 64 * c->H;
-    CKC(cudaMalloc(&c->d_ligx, sizeof(float4) * n_lig), "alloc ligand");
-    CKC(cudaMalloc(&c->d_ligp, sizeof(float4) * n_lig), "alloc ligand");
-    CKC(cudaMalloc(&c->d_lig_rank, sizeof(int) * n_lig), "alloc ligand");
-    CKC(cudaMemcpy(c->d_ligx, lx.data(), sizeof(float4) * n_lig, cudaMemcpyHostToDevice), "H2D ligand");
-    CKC(cudaMemcpy(c->d_ligp, lp.data(), sizeof(float4) * n_lig, cudaMemcpyHostToDevice), "H2D ligand");
-    CKC(cudaMemcpy(c->d_lig_rank, rank.data(), sizeof(int) * n_lig, cudaMemcpyHostToDevice), "H2D ligand");
+    CKC(pool::alloc(&c->d_ligx, sizeof(float4) * n_lig), "alloc ligand");
+    CKC(pool::alloc(&c->d_ligp, sizeof(float4) * n_lig), "alloc ligand");
+    CKC(pool::alloc(&c->d_lig_rank, sizeof(int) * n_lig), "alloc ligand");
+    CKC(cudaMemcpyAsync(c->d_ligx, lx.data(), sizeof(float4) * n_lig, cudaMemcpyHostToDevice, c->stream), "H2D ligand");
+    CKC(cudaMemcpyAsync(c->d_ligp, lp.data(), sizeof(float4) * n_lig, cudaMemcpyHostToDevice, c->stream), "H2D ligand");
+    CKC(cudaMemcpyAsync(c->d_lig_rank, rank.data(), sizeof(int) * n_lig, cudaMemcpyHostToDevice, c->stream), "H2D ligand");
   }
 
   // receptor atoms (absolute) + per-atom parameters
@@ -810,19 +923,20 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   float4* d_prm = nullptr;
   float4* d_centres = nullptr;
   auto free_tmp = [&]() {
-    if (d_rec) cudaFree(d_rec);
-    if (d_prm) cudaFree(d_prm);
-    if (d_centres) cudaFree(d_centres);
+    cudaStreamSynchronize(c->stream);  // list-building launches may still read the temporaries
+    if (d_rec) pool::release(d_rec);
+    if (d_prm) pool::release(d_prm);
+    if (d_centres) pool::release(d_centres);
   };
 #define CKT(expr, where)                                                       \
   do {                                                                         \
     cudaError_t e_ = (expr);                                                   \
     if (e_ != cudaSuccess) { free_tmp(); return fail(cuda_fail(nullptr, e_, where)); } \
   } while (0)
-  CKT(cudaMalloc(&d_rec, sizeof(float4) * n_rec), "alloc receptor");
-  CKT(cudaMalloc(&d_prm, sizeof(float4) * n_rec), "alloc receptor");
-  CKT(cudaMemcpy(d_rec, hrec.data(), sizeof(float4) * n_rec, cudaMemcpyHostToDevice), "H2D receptor");
-  CKT(cudaMemcpy(d_prm, hprm.data(), sizeof(float4) * n_rec, cudaMemcpyHostToDevice), "H2D receptor");
+  CKT(pool::alloc(&d_rec, sizeof(float4) * n_rec), "alloc receptor");
+  CKT(pool::alloc(&d_prm, sizeof(float4) * n_rec), "alloc receptor");
+  CKT(cudaMemcpyAsync(d_rec, hrec.data(), sizeof(float4) * n_rec, cudaMemcpyHostToDevice, c->stream), "H2D receptor");
+  CKT(cudaMemcpyAsync(d_prm, hprm.data(), sizeof(float4) * n_rec, cudaMemcpyHostToDevice, c->stream), "H2D receptor");
 
   std::vector<int> h_off(n_spots), h_len(n_spots), iota(n_spots);
   std::vector<float4> h_shift(n_spots);
@@ -832,8 +946,8 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     // the same relative frame as the cutoff lists: keeps the pair differences accurate)
     std::vector<float4> hc(n_spots);
     for (int s = 0; s < n_spots; ++s) hc[s] = make_float4(spot_xyz[3 * s], spot_xyz[3 * s + 1], spot_xyz[3 * s + 2], 0.0f);
-    CKT(cudaMalloc(&d_centres, sizeof(float4) * n_spots), "alloc");
-    CKT(cudaMemcpy(d_centres, hc.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
+    CKT(pool::alloc(&d_centres, sizeof(float4) * n_spots), "alloc");
+    CKT(cudaMemcpyAsync(d_centres, hc.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
     const int64_t tot = (int64_t)n_rec * n_spots;
     if (tot > 0x7fffffff) { free_tmp(); return fail(set_err(VS_ERR_OUT_OF_MEMORY, "receptor lists exceed 2^31 atoms")); }
     for (int s = 0; s < n_spots; ++s) {
@@ -841,9 +955,9 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
       h_len[s] = n_rec;
       h_shift[s] = make_float4(0, 0, 0, 0);
     }
-    CKT(cudaMalloc(&c->d_lists, sizeof(RecAtom) * tot), "alloc lists");
-    CKT(cudaMalloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
-    CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+    CKT(pool::alloc(&c->d_lists, sizeof(RecAtom) * tot), "alloc lists");
+    CKT(pool::alloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
+    CKT(cudaMemcpyAsync(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
     CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, INFINITY, c->d_list_off, nullptr, c->d_lists, 0,
                            c->stream), "list fill launch");
     c->list_total = tot;
@@ -852,10 +966,10 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     const double reach = (double)c->T * std::sqrt(3.0) + rmax + (double)sp.cutoff + 0.01;
     std::vector<float4> hc(n_spots);
     for (int s = 0; s < n_spots; ++s) hc[s] = make_float4(spot_xyz[3 * s], spot_xyz[3 * s + 1], spot_xyz[3 * s + 2], 0.0f);
-    CKT(cudaMalloc(&d_centres, sizeof(float4) * n_spots), "alloc");
-    CKT(cudaMemcpy(d_centres, hc.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
-    CKT(cudaMalloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
-    CKT(cudaMalloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
+    CKT(pool::alloc(&d_centres, sizeof(float4) * n_spots), "alloc");
+    CKT(cudaMemcpyAsync(d_centres, hc.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
+    CKT(pool::alloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
+    CKT(pool::alloc(&c->d_list_off, sizeof(int) * n_spots), "alloc");
     CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, (float)(reach * reach), nullptr, c->d_list_len,
                            nullptr, 1, c->stream), "list count launch");
     CKT(cudaMemcpyAsync(h_len.data(), c->d_list_len, sizeof(int) * n_spots, cudaMemcpyDeviceToHost, c->stream), "D2H");
@@ -868,36 +982,36 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     }
     if (tot > 0x7fffffff) { free_tmp(); return fail(set_err(VS_ERR_OUT_OF_MEMORY, "receptor lists exceed 2^31 atoms")); }
     c->list_total = tot;
-    CKT(cudaMalloc(&c->d_lists, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
-    CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+    CKT(pool::alloc(&c->d_lists, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
+    CKT(cudaMemcpyAsync(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
     CKT(launch_build_lists(d_rec, d_prm, n_rec, d_centres, n_spots, (float)(reach * reach), c->d_list_off, nullptr,
                            c->d_lists, 0, c->stream), "list fill launch");
     // cell-sorted lists + cell start table (per-chunk culling in the pair kernel)
     CKT(cudaMemcpyAsync(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
     RecAtom* sorted = nullptr;
-    CKT(cudaMalloc(&sorted, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
+    CKT(pool::alloc(&sorted, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
     c->cR = (float)reach + 0.01f;
     c->ch = 2.0f * c->cR / (float)CELL_G;
     c->cinv_h = (float)CELL_G / (2.0f * c->cR);
-    CKT(cudaMalloc(&c->d_cells, sizeof(uint16_t) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
+    CKT(pool::alloc(&c->d_cells, sizeof(uint16_t) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
     cudaError_t es = launch_cell_sort(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_cells, c->cR,
                                       c->cinv_h, c->stream);
     if (es == cudaSuccess) es = cudaStreamSynchronize(c->stream);
-    cudaFree(c->d_lists);
+    pool::release(c->d_lists);
     c->d_lists = sorted;
     CKT(es, "list sort launch");
   }
-  if (!c->d_list_len) CKT(cudaMalloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
-  CKT(cudaMemcpy(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
-  CKT(cudaMemcpy(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
+  if (!c->d_list_len) CKT(pool::alloc(&c->d_list_len, sizeof(int) * n_spots), "alloc");
+  CKT(cudaMemcpyAsync(c->d_list_len, h_len.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
+  CKT(cudaMemcpyAsync(c->d_list_off, h_off.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
   c->W = c->T + (float)rmax + 0.01f;  // cutoff mode: |x_k| <= T + max|l_i| for every transformed atom
   c->inv_hm = (float)(1 << MORTON_BITS) / (2.0f * c->W);
-  CKT(cudaMalloc(&c->d_shift, sizeof(float4) * n_spots), "alloc");
-  CKT(cudaMemcpy(c->d_shift, h_shift.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice), "H2D");
-  CKT(cudaMalloc(&c->d_iota, sizeof(int) * n_spots), "alloc");
-  CKT(cudaMemcpy(c->d_iota, iota.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice), "H2D");
-  CKT(cudaMalloc(&c->d_counters, sizeof(unsigned long long) * 3), "alloc");
-  CKT(cudaMalloc(&c->d_seed, sizeof(uint64_t)), "alloc");
+  CKT(pool::alloc(&c->d_shift, sizeof(float4) * n_spots), "alloc");
+  CKT(cudaMemcpyAsync(c->d_shift, h_shift.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
+  CKT(pool::alloc(&c->d_iota, sizeof(int) * n_spots), "alloc");
+  CKT(cudaMemcpyAsync(c->d_iota, iota.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
+  CKT(pool::alloc(&c->d_counters, sizeof(unsigned long long) * 3), "alloc");
+  CKT(pool::alloc(&c->d_seed, sizeof(uint64_t)), "alloc");
   {
     const char* gv = std::getenv("VS_GRAPHS");
     c->graphs = !(gv && gv[0] == '0');
@@ -997,25 +1111,47 @@ vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t
   return run_impl(c, mp, seed, n_sel, spot_ids, d_best_pose, d_best_score, (cudaStream_t)stream, nullptr);
 }
 
+// VS_DEBUG_TIMING=1: phase times of vs_destroy on stderr (host-side cost investigation)
+static bool debug_timing() {
+  static const bool on = std::getenv("VS_DEBUG_TIMING") != nullptr;
+  return on;
+}
+
 void vs_destroy(vs_ctx* c) {
   if (!c) return;
   DeviceGuard guard(c->dev);
+  using clk = std::chrono::steady_clock;
+  auto t = clk::now();
+  double ph[6] = {0, 0, 0, 0, 0, 0};
+  auto lap = [&](int i) {
+    const auto n = clk::now();
+    ph[i] = std::chrono::duration<double, std::milli>(n - t).count();
+    t = n;
+  };
   if (c->stream) cudaStreamSynchronize(c->stream);
   cudaDeviceSynchronize();
+  lap(0);
   for (auto& b : c->buf) b.release();
+  lap(1);
   for (auto e : c->ev) cudaEventDestroy(e);
   if (c->gexec) cudaGraphExecDestroy(c->gexec);
+  lap(2);
   void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_iota, c->d_counters,
                   c->d_seed, c->d_cells, c->d_ligx, c->d_ligp, c->d_lig_rank};
   for (void* p : ptrs)
-    if (p) cudaFree(p);
+    if (p) pool::release(p);
+  lap(3);
   if (c->stream) cudaStreamDestroy(c->stream);
   for (int i = 0; i < NSUB; ++i) {
     if (c->sub[i]) cudaStreamDestroy(c->sub[i]);
     if (c->ev_join[i]) cudaEventDestroy(c->ev_join[i]);
   }
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  lap(4);
   delete c;
+  if (debug_timing())
+    std::fprintf(stderr, "vs_destroy ms: sync %.2f bufs %.2f events+graph %.2f frees %.2f streams %.2f\n", ph[0], ph[1],
+                 ph[2], ph[3], ph[4]);
 }
 
 const char* vs_last_error(void) { return g_err.c_str(); }
@@ -1070,13 +1206,13 @@ vs_status vs_debug_philox(int64_t n, const uint32_t* ctr, const uint32_t* key, u
   if (n == 0) return VS_OK;
   vs_ctx* c = nullptr;
   uint4 *dc = nullptr, *dout = nullptr;
-  CK(cudaMalloc(&dc, sizeof(uint4) * n), "alloc");
-  cudaError_t e = cudaMalloc(&dout, sizeof(uint4) * n);
+  CK(pool::alloc(&dc, sizeof(uint4) * n), "alloc");
+  cudaError_t e = pool::alloc(&dout, sizeof(uint4) * n);
   if (e == cudaSuccess) e = cudaMemcpy(dc, ctr, sizeof(uint4) * n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = launch_philox(n, dc, make_uint2(key[0], key[1]), dout, nullptr);
   if (e == cudaSuccess) e = cudaMemcpy(out, dout, sizeof(uint4) * n, cudaMemcpyDeviceToHost);
-  cudaFree(dc);
-  if (dout) cudaFree(dout);
+  pool::release(dc);
+  if (dout) pool::release(dout);
   if (e != cudaSuccess) return cuda_fail(c, e, "debug philox");
   return VS_OK;
 }
