@@ -328,6 +328,31 @@ def test_run_deterministic_and_chunk_independent(gpu, oracle_mod):
     np.testing.assert_array_equal(sc, s1[ids])
 
 
+def test_context_churn_bitwise(gpu, oracle_mod):
+    """Contexts created and destroyed back to back, alternating configurations: the device memory cache hands each
+    destroyed context's blocks (with their stale contents) to the next one.  Every run and every scoring call must
+    equal the first one of the same configuration bit for bit, and the first tiny run must match the oracle."""
+    probs = [synth.make_problem("tiny"), synth.make_problem("small")]
+    ref = {}
+    for i in range(6):
+        k = i % 2
+        prob = probs[k]
+        g = vs.Context.from_problem(prob, vs.score_params())
+        mp = vs.mh_preset(3, population=32, generations=3)
+        p, s = g.run(mp, 11)
+        spot, q, t = synth.make_poses(300, prob.cfg.n_spots, 3.0, seed=4)
+        sc = g.score_poses(spot, q, t)
+        g.close()
+        if k not in ref:
+            ref[k] = (p, s, sc)
+            if k == 0:
+                o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params())
+                assert_scores(sc, o.score(spot, q, t), "churn tiny")
+        else:
+            for a, b in zip((p, s, sc), ref[k]):
+                np.testing.assert_array_equal(a, b)
+
+
 def test_run_errors(gpu, oracle_mod):
     prob, (g, _) = _run_pair(oracle_mod)
     with pytest.raises(vs.VSError):
