@@ -154,6 +154,13 @@ VS_API vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, 
                        float* d_best_pose, float* d_best_score, void* cuda_stream);
 
 VS_API void vs_destroy(vs_ctx* c); /* NULL-safe; synchronises the ctx's device work */
+
+/* Device memory of destroyed contexts is cached per device and handed to later contexts of the process (context
+ * create / destroy then cost ~1 ms instead of tens of ms of cudaMalloc / cudaFree).  The cache holds at most
+ * VS_POOL_CACHE_MB MiB per device (environment, read once; default 8192).  vs_release_cached_memory returns the
+ * cached blocks of `cuda_device` (< 0: of every device) to the driver; live contexts keep theirs.  Thread-safe.
+ * Errors: VS_ERR_INVALID_ARGUMENT (no such device). */
+VS_API vs_status vs_release_cached_memory(int32_t cuda_device);
 VS_API const char* vs_last_error(void);
 VS_API int vs_abi_version(void);
 

@@ -1154,6 +1154,23 @@ void vs_destroy(vs_ctx* c) {
                  ph[2], ph[3], ph[4]);
 }
 
+vs_status vs_release_cached_memory(int32_t cuda_device) {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess) n = 0;
+  if (cuda_device >= n) return set_err(VS_ERR_INVALID_ARGUMENT, "no such CUDA device");
+  std::vector<int> devs;
+  {
+    std::lock_guard<std::mutex> g(pool::mu);
+    for (auto& kv : pool::devs())
+      if (cuda_device < 0 || kv.first == cuda_device) devs.push_back(kv.first);
+  }
+  for (int d : devs) {
+    DeviceGuard guard(d);
+    pool::trim(d);
+  }
+  return VS_OK;
+}
+
 const char* vs_last_error(void) { return g_err.c_str(); }
 int vs_abi_version(void) { return VS_ABI_VERSION; }
 

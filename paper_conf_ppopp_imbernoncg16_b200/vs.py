@@ -21,7 +21,16 @@ TRACE_INIT, TRACE_SCORED, TRACE_SELECT, TRACE_LS, TRACE_SORTED, TRACE_COMBINED, 
 # every symbol include/vs.h declares (checked by tests/test_abi.py)
 EXPORTS = ["vs_score_params_default", "vs_mh_preset", "vs_create", "vs_score_poses", "vs_score_poses_device",
            "vs_run", "vs_run_async", "vs_destroy", "vs_last_error", "vs_abi_version", "vs_set_timing",
-           "vs_get_stats", "vs_reset_stats", "vs_list_lengths", "vs_run_trace", "vs_debug_philox"]
+           "vs_get_stats", "vs_reset_stats", "vs_list_lengths", "vs_run_trace", "vs_debug_philox",
+           "vs_release_cached_memory"]
+
+
+def release_cached_memory(device: int = -1) -> None:
+    """Return the device memory cached from destroyed contexts to the driver (vs_release_cached_memory)."""
+    L = load()
+    st = L.vs_release_cached_memory(device)
+    if st != 0:
+        raise VSError(st, L.vs_last_error().decode())
 
 
 class VSError(RuntimeError):
@@ -93,6 +102,8 @@ def load(build_if_stale: bool = True):
     L.vs_run_trace.argtypes = [vp, C.POINTER(MHParams), C.c_uint64, C.c_int32, i32p, f32p, f32p, TRACE_FN, vp]
     L.vs_destroy.argtypes = [vp]
     L.vs_destroy.restype = None
+    L.vs_release_cached_memory.argtypes = [C.c_int32]
+    L.vs_release_cached_memory.restype = C.c_int
     L.vs_last_error.restype = C.c_char_p
     L.vs_abi_version.restype = C.c_int
     L.vs_set_timing.argtypes = [vp, C.c_int]

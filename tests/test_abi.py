@@ -56,6 +56,7 @@ def test_argument_errors_without_device():
     assert b"NULL" in L.vs_last_error()
     assert L.vs_score_poses(None, 1, None, None, None, None) == vs.ERR_INVALID_ARGUMENT
     L.vs_destroy(None)  # NULL-safe
+    assert L.vs_release_cached_memory(1 << 20) == vs.ERR_INVALID_ARGUMENT  # no such device (none at all here)
 
 
 def test_create_without_gpu_fails_loudly():
