@@ -179,7 +179,7 @@ struct DevBuf {
 };
 
 #ifndef VS_NSUB
-#define VS_NSUB 8
+#define VS_NSUB 12
 #endif
 constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
 #ifndef VS_MAX_SPLIT
@@ -194,7 +194,7 @@ static_assert(vsk::CELL_G % MAX_SPLIT == 0, "the pair kernel assigns cell rows t
 #define VS_BIG_RUN_SPOTS 256  // runs of at least this many spots use at most VS_BIG_RUN_GROUPS streams
 #endif
 #ifndef VS_BIG_RUN_GROUPS
-#define VS_BIG_RUN_GROUPS 8
+#define VS_BIG_RUN_GROUPS 12
 #endif
 #ifndef VS_SPLIT_WARPS
 #define VS_SPLIT_WARPS 16     // chunks x splits per spot at least ...
@@ -507,9 +507,10 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
   // Spots are independent: split them into groups whose generation loops run on separate
   // streams, enqueued generation by generation, so one group's kernels fill the wave tails of
   // another's.
-  // Stream count (measured on B200, profiles/r01_notes.md): small runs are chains of latency-bound launches and
-  // gain from every extra stream (64 spots: 4 -> 16 streams, 25.8 -> 23.1 ms / step); large runs fill the GPU
-  // with 8 (500 spots: 8 streams 598 ms, 16 streams 603 ms).
+  // Stream count (measured on B200, profiles/r01_notes.md): runs are chains of partly latency-bound launches and
+  // gain from extra streams (64 spots: 4 -> 8 streams, 25.8 -> 24.6 ms / step; 500 spots: 8 -> 12 streams, with
+  // the pair kernel at 20 CTAs / SM, 564 -> 553 ms / step), but every stream adds launches to a context's first,
+  // un-graphed run (host-bound: 16 streams doubled it on the small config), hence >= 8 spots per group.
   int G = std::max(1, std::min(NSUB, ns / VS_GROUP_SPOTS));
   if (ns >= VS_BIG_RUN_SPOTS) G = std::min(G, VS_BIG_RUN_GROUPS);
   if (tr) G = 1;
