@@ -125,6 +125,17 @@ class ClockSampler:
         return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
 
 
+def cpu_model() -> str:
+    """The host CPU model (the oracle timing states the cores and the CPU model)."""
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -208,7 +219,8 @@ def run_reference(args, rank, world):
         "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
         "config": {"workload": args.config, "preset": f"M{args.preset}", "mode": args.mode, "sample": sample},
         "poses_per_s": poses / (ms * 1e-3),
-        "cpu_baseline": {"value": val, "unit": "pairs/s", "cores": cores, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": val, "unit": "pairs/s", "cores": cores, "cpu": cpu_model(), "kind": "oracle",
+                         "sample": sample},
         "e2e": {"value": val, "unit": "pairs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
@@ -465,7 +477,7 @@ def main():
         dt, pr, po, cores = oracle_sample(prob, {"cutoff": cutoff},
                                           {"preset": args.preset, "population": cfg.population}, lens,
                                           args.seed, n_s, Gs)
-        cpu = {"value": pr / dt, "unit": "pairs/s", "cores": cores, "kind": "oracle",
+        cpu = {"value": pr / dt, "unit": "pairs/s", "cores": cores, "cpu": cpu_model(), "kind": "oracle",
                "sample": f"fp64 oracle vso_run, {n_s} spots x {Gs} generations of {args.config} "
                          f"(P={cfg.population}, M{args.preset}), {po} poses, {dt:.1f} s; pairs counted as the "
                          f"workload defines them (n_lig x list length), the oracle itself visits all n_rec atoms"}
