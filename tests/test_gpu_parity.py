@@ -249,8 +249,8 @@ def test_device_entry_point(gpu, oracle_mod):
 def test_stats_count_pairs(gpu, oracle_mod):
     """`pairs` = workload pairs, n_lig x list length of the pose's spot per scored pose (the whole receptor in
     all-pairs mode); `pairs_evaluated` = item slots x receptor atoms streamed per chunk: every list atom in
-    all-pairs mode (plus the padding slots of a chunk), in cutoff mode only the cell rows within rc of a
-    chunk's bounding box."""
+    all-pairs mode (plus the padding slots of a chunk), in cutoff mode only the atoms of the cell rows within rc
+    of a chunk's bounding box that are also within rc of the bounding box of the item's slot pair."""
     prob = synth.make_problem("tiny")
     spot, q, t = synth.make_poses(100, 4, 3.0, seed=2)
     g, _ = both(oracle_mod, prob, 0.0)
