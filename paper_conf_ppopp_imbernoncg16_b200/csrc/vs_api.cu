@@ -879,10 +879,18 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     std::vector<float4> lx(n_lig), lp(n_lig);
     std::vector<int> rank(n_lig);
     int cnt[2] = {0, 0};
+    bool any_role = false;  // a ligand without H-bond atoms keeps H = 0 (no H-bond slots) even with VS_CELL_MERGE
+    for (int i = 0; i < n_lig; ++i) any_role = any_role || don[lig_type[i]] != 0.0f || acc[lig_type[i]] != 0.0f;
+    const bool merge = VS_CELL_MERGE && any_role;
     for (int i = 0; i < n_lig; ++i) {
       const int t = lig_type[i];
-      const int cls = (don[t] != 0.0f || acc[t] != 0.0f) ? 1 : 0;
-      lx[i] = make_float4(lig_xyz[3 * i] - cen[0], lig_xyz[3 * i + 1] - cen[1], lig_xyz[3 * i + 2] - cen[2], (float)cls);
+      const int role = (don[t] != 0.0f || acc[t] != 0.0f) ? 1 : 0;
+      // item class (K1 sorts and chunks the classes apart; class-1 items sit in H-bond slots): the H-bond role, or
+      // class 1 for every atom with VS_CELL_MERGE (one curve order for all items, all slots H-bond slots).  ligx.w
+      // = 0 class 0; 1 class 1 with an H-bond role; 2 class 1 without one (its H-bond sums are discarded)
+      const int cls = merge ? 1 : role;
+      lx[i] = make_float4(lig_xyz[3 * i] - cen[0], lig_xyz[3 * i + 1] - cen[1], lig_xyz[3 * i + 2] - cen[2],
+                          cls == 0 ? 0.0f : (role ? 1.0f : 2.0f));
       const double qk = sp.dielectric == 0 ? (double)sp.coulomb_k * lig_q[i] / 4.0
                                            : (double)sp.coulomb_k * lig_q[i] / (double)sp.eps_r;
       lp[i] = make_float4((float)qk, c12[t], c6[t], don[t]);
@@ -894,7 +902,7 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     // with 19 slots per class-0-only pair and 23 per H-bond pair; class-0 items may overflow
     // into H-bond slots, so chunks per pose = max(n / CH_ITEMS, nh / (64 H))
     double best = 1e300;
-    for (int h = 0; h <= CELL_KP; ++h) {
+    for (int h = merge ? CELL_KP : 0; h <= CELL_KP; ++h) {
       if (c->nh > 0 && h == 0) continue;
       const double per = std::max((double)n_lig / CH_ITEMS, h > 0 ? c->nh / (64.0 * h) : 0.0);
       const double cost = per * (19.0 * (CELL_KP - h) + 23.0 * h);

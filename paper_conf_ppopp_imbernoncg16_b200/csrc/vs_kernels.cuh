@@ -56,6 +56,9 @@ enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
 // Work unit = chunk of up to CH_ITEMS transformed ligand atoms ("items": one ligand atom of one pose),
 // spatially sorted per spot; the chunk streams only the cell rows of the spot's cell-sorted list
 // within rc of its bounding box.
+#ifndef VS_CELL_MERGE
+#define VS_CELL_MERGE 0  // 1: every ligand atom in class 1 (one item order, all slot pairs H-bond pairs)
+#endif
 #ifndef VS_CELL_G
 #define VS_CELL_G 24
 #endif
@@ -87,7 +90,7 @@ struct CellArgs {
   const uint16_t* cells;
   float cR, ch, cinv_h;      // grid half-width (A), cell edge, 1 / edge
   // ligand (input order)
-  const float4* ligx;        // local x, y, z (centred), w = class (0: no H-bond role, 1: donor / acceptor)
+  const float4* ligx;        // local x, y, z (centred), w = class (0: class 0; 1: class 1, donor / acceptor; 2: class 1, no role)
   const float4* ligp;        // es_i, c12_i, c6_i, donor_i
   const int* lig_rank;       // rank of the atom within its class
   int n_lig, nn, nh;         // atoms, of which nn without / nh with an H-bond role
