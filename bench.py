@@ -169,9 +169,10 @@ def oracle_sample(prob, sp_kw, mp_kw, list_len, seed, n_spots_sample: int, gener
     t0 = time.perf_counter()
     o.run(mp, seed, ids)
     dt = time.perf_counter() - t0
-    poses = o.pairs_evaluated() // (prob.cfg.n_lig * prob.cfg.n_rec)
+    n_lig = len(prob.lig.q)      # the sampled ligand (sweep: ligand 0; cfg.n_lig is per-ligand there)
+    poses = o.pairs_evaluated() // (n_lig * prob.cfg.n_rec)
     per_spot = poses // n_spots_sample
-    pairs = int(sum(int(list_len[s]) for s in ids)) * prob.cfg.n_lig * per_spot
+    pairs = int(sum(int(list_len[s]) for s in ids)) * n_lig * per_spot
     return dt, pairs, poses, min(n_spots_sample, oracle.get_threads())
 
 
@@ -471,6 +472,7 @@ def main():
         lens = ctx.list_lengths()
         if sweep:
             prob.lig = prob.ligands[0]
+            lens = list_lengths_host(prob, cutoff)     # ligand 0's lists (the sampled ligand)
         import oracle
         n_s = max(1, min(n_spots, oracle.get_threads()))
         Gs = 2 if args.config in ("medium", "large", "sweep") else min(G, 5)

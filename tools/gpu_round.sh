@@ -2,7 +2,7 @@
 # One GPU measurement pass of the current build (run under gpurun from the repo root):
 # GPU tests, bench lines (medium default, small, large), ncu launch list and a full capture of the pair kernel.
 set -x
-O=${OUT:-gpurun_out/r01s4}
+O=${OUT:-gpurun_out/r01s5}
 mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > $O/smi.txt 2>&1
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log
