@@ -46,3 +46,19 @@ def test_bench_two_ranks_gloo_on_one_gpu(scaling):
               "bench.py", "--gpus", "2", "--config", "small", "--steps", "1", "--warmup", "3", "--generations", "3",
               "--scaling", scaling, "--no-micro", "--no-cpu-baseline"], env={"VS_BENCH_BACKEND": "gloo"})
     assert d["n_gpus"] == 2 and d["scaling"] == scaling and d["value"] > 0
+
+
+def test_cpu_baseline_sample_sweep_library():
+    """The cpu_baseline leg samples ligand 0 of a screening library (cfg.n_lig is 0 there): the pair count is
+    n_lig(ligand 0) x list length x poses per spot, and the pose count is population x (1 + generations x steps)."""
+    sys.path.insert(0, ROOT)
+    import bench
+    from paper_conf_ppopp_imbernoncg16_b200 import synth
+    prob = synth.make_problem("sweep")
+    assert prob.cfg.n_lig == 0
+    prob.lig = prob.ligands[0]
+    lens = bench.list_lengths_host(prob, 12.0)
+    dt, pairs, poses, cores = bench.oracle_sample(prob, {"cutoff": 12.0}, {"preset": 3, "population": 64},
+                                                  lens, 0, 2, 1)
+    assert dt > 0 and cores >= 1 and poses > 0 and poses % 2 == 0
+    assert pairs == (int(lens[0]) + int(lens[1])) * len(prob.lig.q) * (poses // 2)
