@@ -481,7 +481,8 @@ def main():
             lens = list_lengths_host(prob, cutoff)     # ligand 0's lists (the sampled ligand)
         import oracle
         n_s = max(1, min(n_spots, oracle.get_threads()))
-        Gs = 2 if args.config in ("medium", "large", "sweep") else min(G, 5)
+        # generations in the sample: about 10 s of oracle work on 16 host threads
+        Gs = min(G, {"medium": 10, "large": 4, "sweep": 40}.get(args.config, 50))
         dt, pr, po, cores = oracle_sample(prob, {"cutoff": cutoff},
                                           {"preset": args.preset, "population": cfg.population}, lens,
                                           args.seed, n_s, Gs)
