@@ -86,6 +86,8 @@ def lib():
                                       C.c_int32, f32p, f32p]
         L.vso_ls_proposal_k.argtypes = [vp, C.POINTER(MHParams), C.c_uint64, C.c_int32, C.c_int32, C.c_int32,
                                         C.c_int32, C.c_int32, f32p, f32p]
+        L.vso_select_parents.argtypes = [C.POINTER(MHParams), C.c_uint64, C.c_int32, C.c_int32, C.c_int32,
+                                         i32p, i32p]
         L.vso_improve_count.argtypes = [C.POINTER(MHParams)]
         L.vso_select_improve.argtypes = [f64p, C.c_int32, C.c_int32, i32p]
         L.vso_include.argtypes = [f64p, f64p, C.c_int32, i32p]
@@ -157,6 +159,13 @@ def select_improve(scores, m: int) -> np.ndarray:
     J = np.zeros(m, dtype=np.int32)
     lib().vso_select_improve(_p(s, C.c_double), len(s), m, _p(J, C.c_int32))
     return J
+
+
+def select_parents(mp: MHParams, seed: int, spot: int, g: int, j: int) -> tuple[int, int]:
+    """Select (R13): sorted-population ranks of the two parents of child j."""
+    a, b = C.c_int32(), C.c_int32()
+    lib().vso_select_parents(C.byref(mp), seed, spot, g, j, C.byref(a), C.byref(b))
+    return a.value, b.value
 
 
 def include(sS, sC) -> np.ndarray:

@@ -630,6 +630,15 @@ void vso_combine_child(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed,
   from_pose(o, out);
 }
 
+void vso_select_parents(const vso_mh_params* mp, uint64_t seed, int32_t spot, int32_t g, int32_t j,
+                        int32_t* p1_out, int32_t* p2_out) {
+  MH mh{nullptr, *mp, seed, spot, 1};
+  int p1, p2;
+  mh.select(g, j, p1, p2);
+  *p1_out = p1;
+  *p2_out = p2;
+}
+
 void vso_ls_proposal(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot, int32_t g,
                      int32_t l, int32_t j, const float in[7], float out[7]) {
   vso_ls_proposal_k(c, mp, seed, spot, g, l, 0, j, in, out);

@@ -78,6 +78,9 @@ uint64_t vso_pairs_evaluated(const vso_ctx* c);   /* running count of (i,j) pair
 void vso_init_pose(const vso_ctx* c, uint64_t seed, int32_t spot, int32_t i, float pose_out[7]);
 void vso_combine_child(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot,
                        int32_t g, int32_t j, const float* S_sorted /*[P][7]*/, float pose_out[7]);
+/* Select (R13): the parents (sorted-population ranks) of child j of generation g at `spot` */
+void vso_select_parents(const vso_mh_params* mp, uint64_t seed, int32_t spot, int32_t g, int32_t j,
+                        int32_t* p1_out, int32_t* p2_out);
 void vso_ls_proposal(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot,
                      int32_t g, int32_t l, int32_t j, const float pose_in[7], float pose_out[7]);
 /* proposal k (0 <= k < ls_neighbours) of Improve step l for individual j */
