@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define VS_ABI_VERSION 3
+#define VS_ABI_VERSION 4
 
 #if defined(__GNUC__)
 #define VS_API __attribute__((visibility("default")))
@@ -78,11 +78,20 @@ typedef struct {
   const float* type_sigma;    /* [n_types] A   (>= 0) */
   const float* type_eps;      /* [n_types] kcal/mol (>= 0) */
   const int* type_hb_role;    /* [n_types] 0 none, 1 donor, 2 acceptor */
+  int list_splits;            /* canonical receptor-list splits S: 1, 2 or 4; 0 (default) = by the spot count
+                                 (<= 128 spots: 4, <= 256: 2, else 1).  The GPU sums each
+                                 split's pairs in fp32 and combines the split energies of an atom by the fixed fp64
+                                 tree (e0 + e1) + (e2 + e3): a summation order, so scores differ from S = 1 at fp32
+                                 rounding (all within the tolerance).  For a given S a pose's score is the same from
+                                 every entry point and launch, whatever the spot count or GPU count of the run; S > 1
+                                 gives latency-bound runs (few spots per GPU) up to S x more parallel work.  Not
+                                 part of the method: the oracle ignores it. */
 } vs_score_params;
 
 /* Metaheuristic parameters (Algorithm 1; Table 4).
  * population P (1..2048; >= 2 when generations > 0), generations G >= 0
- * (End condition, R20), ls_steps L >= 0 (Improve, R16), improve_frac f in
+ * (End condition, R20), ls_steps L >= 0 with L x ls_neighbours <= 2^23
+ * (the LS Philox counter, R23) (Improve, R16), improve_frac f in
  * [0,1] (Table 4 "% of elements to be improved"; m = clamp(round(f*P),1,P)
  * elements, R17), p_mut in [0,1] (R15), step sizes >= 0 (A, radians-ish
  * quaternion increments). */
@@ -131,9 +140,13 @@ VS_API vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32
 VS_API vs_status vs_score_poses(vs_ctx* c, int64_t n, const int32_t* spot, const float* quat_wxyz, const float* trans,
                          float* score_out);
 
-/* Same on device buffers, asynchronous on `cuda_stream` (a cudaStream_t;
- * NULL = legacy default stream).  Poses that fail validation get a NaN
- * score instead of an error status (no host round trip). */
+/* Same on device buffers, asynchronous with respect to `cuda_stream` (a
+ * cudaStream_t; NULL = legacy default stream): the work is ordered after
+ * everything enqueued on `cuda_stream` before the call, and later work on
+ * `cuda_stream` is ordered after it (it runs on the ctx's own stream, joined
+ * by events, so calls of one ctx never overlap each other, whatever streams
+ * the caller uses).  Poses that fail validation get a NaN score instead of
+ * an error status (no host round trip). */
 VS_API vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_spot, const float* d_quat,
                                 const float* d_trans, float* d_score, void* cuda_stream);
 
@@ -147,9 +160,12 @@ VS_API vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_sp
 VS_API vs_status vs_run(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
                  float* best_pose_out, float* best_score_out);
 
-/* Same, asynchronous on `cuda_stream`; outputs in device memory.  spot_ids
- * is a HOST array (validated on the host).  The ctx's workspace is reused:
- * do not overlap two vs_run_async calls of one ctx on different streams. */
+/* Same, asynchronous with respect to `cuda_stream` (ordered after prior work
+ * on it, later work on it ordered after the run; NULL = legacy default
+ * stream); outputs in device memory.  spot_ids is a HOST array (validated
+ * on the host, copied before the call returns).  The run itself executes on
+ * the ctx's own streams (a CUDA graph from the second identical call on), so
+ * calls of one ctx are serialised whatever streams the caller passes. */
 VS_API vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
                        float* d_best_pose, float* d_best_score, void* cuda_stream);
 
@@ -172,12 +188,27 @@ typedef struct {
   uint64_t pairs;            /* workload atom pairs: n_lig x list length (n_rec in all-pairs mode) per scored pose */
   double score_ms;           /* summed CUDA-event time of scoring launches (timing enabled) */
   uint64_t timed_launches;   /* launches covered by score_ms */
-  uint64_t pairs_evaluated;  /* pairs the pair kernel evaluated: item slots x receptor atoms streamed per chunk
-                                (<= pairs in cutoff mode: cell culling skips list atoms beyond rc of a chunk) */
+  uint64_t pairs_evaluated;  /* pairs the pair kernel evaluated: item slots x receptor atoms swept for them
+                                (< pairs in cutoff mode: cell and slot-pair culling skip atoms beyond rc) */
+  uint64_t pairs_within;     /* pairs within the cutoff, r^2 < rc^2 (census launches only, VS_TIMING_CENSUS):
+                                the interactions that contribute to the scores; all-pairs mode: = pairs */
+  double pair_busy_ms;       /* VS_TIMING_KERNEL: length of the union of the pair kernel's launch intervals */
+  double pair_launch_ms;     /* VS_TIMING_KERNEL: sum of the pair kernel's launch intervals (first warp start to
+                                last warp end, device globaltimer; concurrent launches overlap) */
+  uint64_t pair_timed_launches;
 } vs_stats;
 
-/* enable = 1: bracket every scoring launch with CUDA events on its stream. */
-VS_API vs_status vs_set_timing(vs_ctx* c, int enable);
+/* Instrumentation flags of vs_set_timing (OR-ed):
+ *   VS_TIMING_EVENTS  CUDA events around every scoring call of direct (un-graphed) launches -> score_ms;
+ *   VS_TIMING_KERNEL  the pair kernel records its launch interval (first warp start, last warp end) on the
+ *                     device globaltimer, also inside replayed CUDA graphs -> pair_busy_ms, pair_launch_ms;
+ *   VS_TIMING_CENSUS  pair-kernel launches count the pairs within rc (another instantiation of the same
+ *                     arithmetic: scores are bitwise unchanged) -> pairs_within.
+ * Changing the flags selects another CUDA graph of vs_run. */
+#define VS_TIMING_EVENTS 1
+#define VS_TIMING_KERNEL 2
+#define VS_TIMING_CENSUS 4
+VS_API vs_status vs_set_timing(vs_ctx* c, int flags);
 /* Synchronises the ctx's device and returns counters since the last reset. */
 VS_API vs_status vs_get_stats(vs_ctx* c, vs_stats* out);
 VS_API vs_status vs_reset_stats(vs_ctx* c);

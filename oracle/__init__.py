@@ -79,6 +79,8 @@ def lib():
         L.vso_ligand_local.argtypes = [vp, f32p]
         L.vso_pairs_evaluated.argtypes = [vp]
         L.vso_pairs_evaluated.restype = C.c_uint64
+        L.vso_pairs_within.argtypes = [vp]
+        L.vso_pairs_within.restype = C.c_uint64
         L.vso_init_pose.argtypes = [vp, C.c_uint64, C.c_int32, C.c_int32, f32p]
         L.vso_combine_child.argtypes = [vp, C.POINTER(MHParams), C.c_uint64, C.c_int32, C.c_int32, C.c_int32,
                                         f32p, f32p]
@@ -245,6 +247,10 @@ class Oracle:
 
     def pairs_evaluated(self) -> int:
         return lib().vso_pairs_evaluated(self.h)
+
+    def pairs_within(self) -> int:
+        """Visited pairs with r^2 < rc^2 (every pair in all-pairs mode): the interactions that contribute."""
+        return lib().vso_pairs_within(self.h)
 
     # ---- lockstep building blocks (pose = 7 floats) ----
     def init_pose(self, seed: int, spot: int, i: int) -> np.ndarray:

@@ -66,6 +66,7 @@ struct vso_ctx {
   std::vector<int> role;
   double hb_C, hb_D;
   std::atomic<uint64_t> pairs{0};
+  std::atomic<uint64_t> pairs_within{0};  // pairs inside the cutoff (instrumentation)
 };
 
 namespace {
@@ -216,6 +217,7 @@ double score_pose(const vso_ctx* c, int s, const float qf[4], const float tf[3])
       {s2 * (x * y + w * z), 1.0 - s2 * (x * x + z * z), s2 * (y * z - w * x)},
       {s2 * (x * z - w * y), s2 * (y * z + w * x), 1.0 - s2 * (x * x + y * y)}};
   double total = 0.0;
+  uint64_t within = 0;  // instrumentation: pairs inside the cutoff (all pairs in all-pairs mode)
   for (int i = 0; i < c->n_lig; ++i) {
     double l[3] = {c->lig_local[3 * i], c->lig_local[3 * i + 1], c->lig_local[3 * i + 2]};
     double xi[3];
@@ -225,9 +227,11 @@ double score_pose(const vso_ctx* c, int s, const float qf[4], const float tf[3])
       double dx = xi[0] - c->rec_xyz[3 * j], dy = xi[1] - c->rec_xyz[3 * j + 1], dz = xi[2] - c->rec_xyz[3 * j + 2];
       double r2 = dx * dx + dy * dy + dz * dz;
       total += pair_energy(c, c->lig_type[i], c->lig_q[i], c->rec_type[j], c->rec_q[j], r2);
+      within += c->all_pairs || std::max(r2, c->r2min) < c->rc * c->rc;
     }
   }
   const_cast<vso_ctx*>(c)->pairs.fetch_add((uint64_t)c->n_lig * (uint64_t)c->n_rec, std::memory_order_relaxed);
+  const_cast<vso_ctx*>(c)->pairs_within.fetch_add(within, std::memory_order_relaxed);
   return total;
 }
 
@@ -375,6 +379,9 @@ vso_status check_mh(const vso_mh_params* mp) {
   if (mp->generations > 0 && mp->population < 2) return fail(VSO_ERR_INVALID_ARGUMENT, "population must be >= 2 when generations > 0");
   if (mp->ls_steps < 0) return fail(VSO_ERR_INVALID_ARGUMENT, "ls_steps must be >= 0");
   if (mp->ls_neighbours < 1 || mp->ls_neighbours > 64) return fail(VSO_ERR_INVALID_ARGUMENT, "ls_neighbours must be in [1, 64]");
+  // LS counter word (TAG_LS << 24) | (2 (l K + k) + 1) stays below 2^24 (R23)
+  if ((long long)mp->ls_steps * mp->ls_neighbours > (1ll << 23))
+    return fail(VSO_ERR_INVALID_ARGUMENT, "ls_steps x ls_neighbours must be <= 2^23");
   if (!(mp->improve_frac >= 0.0f && mp->improve_frac <= 1.0f)) return fail(VSO_ERR_INVALID_ARGUMENT, "improve_frac must be in [0, 1]");
   if (!(mp->p_mut >= 0.0f && mp->p_mut <= 1.0f)) return fail(VSO_ERR_INVALID_ARGUMENT, "p_mut must be in [0, 1]");
   const float st[4] = {mp->mut_trans, mp->mut_rot, mp->ls_trans, mp->ls_rot};
@@ -600,6 +607,7 @@ void vso_ligand_local(const vso_ctx* c, float* out) {
 }
 
 uint64_t vso_pairs_evaluated(const vso_ctx* c) { return c->pairs.load(); }
+uint64_t vso_pairs_within(const vso_ctx* c) { return c->pairs_within.load(); }
 
 static void to_pose(const float in[7], Pose& p) {
   for (int a = 0; a < 4; ++a) p.q[a] = in[a];

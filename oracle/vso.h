@@ -74,6 +74,7 @@ double   vso_score_one(const vso_ctx* c, int32_t spot, const float q[4], const f
 /* ligand coordinates relative to the fp32 centroid, as used by the pose transform */
 void     vso_ligand_local(const vso_ctx* c, float* out_xyz /*[n_lig][3]*/);
 uint64_t vso_pairs_evaluated(const vso_ctx* c);   /* running count of (i,j) pairs visited */
+uint64_t vso_pairs_within(const vso_ctx* c);      /* running count of visited pairs with r^2 < rc^2 (all in all-pairs mode) */
 /* pose = float[7] = (w,x,y,z,tx,ty,tz) */
 void vso_init_pose(const vso_ctx* c, uint64_t seed, int32_t spot, int32_t i, float pose_out[7]);
 void vso_combine_child(const vso_ctx* c, const vso_mh_params* mp, uint64_t seed, int32_t spot,

@@ -4,9 +4,10 @@
 // The paper's host loop copies the candidate set to each GPU and back for
 // every scoring call (Algorithm 2).  Here the whole population
 // lives in HBM for the run; the host only sequences kernel launches (spot
-// groups on up to 4 streams, captured as one CUDA graph on repeated calls),
+// groups on up to 12 streams, captured as one CUDA graph on repeated calls),
 // and the device boundary is crossed at the start (seed, spot ids) and the
 // end (best pose + score per spot).
+#include <algorithm>
 #include <chrono>
 #include <cmath>
 #include <cstdio>
@@ -182,11 +183,7 @@ struct DevBuf {
 #define VS_NSUB 12
 #endif
 constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
-#ifndef VS_MAX_SPLIT
-#define VS_MAX_SPLIT 8
-#endif
-constexpr int MAX_SPLIT = VS_MAX_SPLIT;  // receptor-list splits of one scoring launch (cell_nsplit; a power of 2)
-static_assert(vsk::CELL_G % MAX_SPLIT == 0, "the pair kernel assigns cell rows to splits by cy mod nsplit");
+static_assert(vsk::CELL_G % vsk::CELL_NSPLIT == 0, "the pair kernel assigns cell rows to splits by cy mod NSPLIT");
 #ifndef VS_GROUP_SPOTS
 #define VS_GROUP_SPOTS 8    // spots per stream group at least
 #endif
@@ -196,14 +193,14 @@ static_assert(vsk::CELL_G % MAX_SPLIT == 0, "the pair kernel assigns cell rows t
 #ifndef VS_BIG_RUN_GROUPS
 #define VS_BIG_RUN_GROUPS 12
 #endif
-#ifndef VS_SPLIT_WARPS
-#define VS_SPLIT_WARPS 16     // chunks x splits per spot at least ...
+#ifndef VS_FILL_WARPS
+#define VS_FILL_WARPS 2048    // pair-kernel warps below which a scoring round uses KP = 1 chunks (launch shape)
 #endif
-#ifndef VS_SPLIT_WARPS_MAX
-#define VS_SPLIT_WARPS_MAX 64  // ... raised for contexts with few spots, up to this
+#ifndef VS_GRAPH_CACHE
+#define VS_GRAPH_CACHE 4      // CUDA graphs kept per context
 #endif
-#ifndef VS_SPLIT_TOTAL
-#define VS_SPLIT_TOTAL 4096    // pair-kernel warps a launch over all spots of the context should reach (~1 wave)
+#ifndef VS_KT_CAP
+#define VS_KT_CAP (1 << 20)   // pair-kernel launch intervals kept (instrumentation)
 #endif
 
 enum Buf { B_SEG, B_SA, B_SB, B_C, B_J, B_SPOT, B_Q, B_T, B_OUT, B_VALID, B_COUNTS, B_PP, B_BP, B_CUR,
@@ -231,33 +228,45 @@ struct vs_ctx {
   int* d_list_len = nullptr;
   float4* d_shift = nullptr;
   int* d_iota = nullptr;
-  unsigned long long* d_counters = nullptr;  // [0] pairs evaluated, [1] poses, [2] workload pairs
+  unsigned long long* d_counters = nullptr;  // [0] pairs evaluated, [1] poses, [2] workload pairs, [3] within rc
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
   uint16_t* d_cells = nullptr;          // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
   float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
-  int split_warps = VS_SPLIT_WARPS;     // cell_nsplit target, fixed at vs_create from n_spots
+  long long fill_warps = VS_FILL_WARPS;  // launch shape target (speed only)
+  int nsplit = 1;                        // canonical receptor-list splits (vs_score_params.list_splits)
+  int force_kp = 0;                      // VS_SHAPE=kp (experiments)
   float4* d_ligx = nullptr;             // [n_lig] centred local coordinates, w = class
   float4* d_ligp = nullptr;             // [n_lig] es, c12, c6, donor
   int* d_lig_rank = nullptr;            // [n_lig] rank within the class
-  int nn = 0, nh = 0, H = 0, cn = 0, chb = 0;
+  int nn = 0, nh = 0, H2 = 0, H1 = 0;  // H-bond slot pairs of the KP = 2 / KP = 1 pair kernels
   float W = 0.0f, inv_hm = 0.0f;
   cudaStream_t stream = nullptr;
   cudaStream_t sub[NSUB] = {};          // per-spot-group streams of vs_run
   cudaEvent_t ev_fork = nullptr, ev_join[NSUB] = {};
+  cudaEvent_t ev_in = nullptr, ev_out = nullptr;  // caller stream <-> ctx stream ordering of the async entry points
   DevBuf buf[B_COUNT];
   bool poisoned = false;
   // instrumentation
   uint64_t launches = 0, score_launches = 0;
-  bool timing = false;
+  bool timing = false, ktime = false, census = false;
+  unsigned long long* d_kt = nullptr;       // [VS_KT_CAP][2] pair-kernel launch intervals (~start, end) in ns
+  unsigned long long* d_kt_base = nullptr;  // first slot of the next run's region
+  int kt_local = 0;                         // slots used by the run being enqueued
   std::vector<cudaEvent_t> ev;  // pairs (start, end)
   size_t ev_used = 0;
   double score_ms_acc = 0.0;
   uint64_t timed_acc = 0;
-  // CUDA graph of vs_run (captured on the second identical call)
+  // CUDA graphs of vs_run: captured on the second identical call, a few kept (LRU) so that runs of a few shapes
+  // (spot-chunk sizes of a multi-GPU queue) all replay
+  struct Graph {
+    unsigned char key[256];
+    cudaGraphExec_t exec = nullptr;
+    uint64_t launches = 0, score_launches = 0, used = 0;
+  };
   bool graphs = true, capturing = false, has_last = false;
-  cudaGraphExec_t gexec = nullptr;
-  unsigned char gkey[256] = {}, last_key[256] = {};
-  uint64_t g_launches = 0, g_score_launches = 0;
+  std::vector<Graph> gcache;
+  uint64_t gclock = 0;
+  unsigned char last_key[256] = {};
 };
 
 namespace {
@@ -285,6 +294,9 @@ vs_status check_mh(const vs_mh_params* mp) {
   if (mp->ls_steps < 0) return set_err(VS_ERR_INVALID_ARGUMENT, "ls_steps must be >= 0");
   if (mp->ls_neighbours < 1 || mp->ls_neighbours > 64)
     return set_err(VS_ERR_INVALID_ARGUMENT, "ls_neighbours must be in [1, 64]");
+  // the LS Philox counter word is (TAG_LS << 24) | (2 (l K + k) + 1): it must stay below 2^24 (R23)
+  if ((long long)mp->ls_steps * mp->ls_neighbours > (1ll << 23))
+    return set_err(VS_ERR_INVALID_ARGUMENT, "ls_steps x ls_neighbours must be <= 2^23");
   if (!(mp->improve_frac >= 0.0f && mp->improve_frac <= 1.0f)) return set_err(VS_ERR_INVALID_ARGUMENT, "improve_frac must be in [0, 1]");
   if (!(mp->p_mut >= 0.0f && mp->p_mut <= 1.0f)) return set_err(VS_ERR_INVALID_ARGUMENT, "p_mut must be in [0, 1]");
   const float st[4] = {mp->mut_trans, mp->mut_rot, mp->ls_trans, mp->ls_rot};
@@ -313,14 +325,39 @@ vs_status collect_timing(vs_ctx* c) {
   return VS_OK;
 }
 
-// list splits of a scoring launch: a spot whose chunks number fewer than split_warps has its cell rows dealt
-// over up to MAX_SPLIT splits.  split_warps is a property of the context (set at vs_create from n_spots: few
-// spots, small launches, more splits), so the choice depends on per-spot quantities and the context only --
-// results stay bitwise identical across spot chunkings of a run and GPU counts.
-int cell_nsplit(int nch, int split_warps) {
-  int ns = 1;
-  while (ns < MAX_SPLIT && (long)nch * ns < split_warps) ns *= 2;
-  return ns;
+// Launch shape of a scoring launch: KP packed item pairs per lane (items per chunk = 64 KP); every chunk takes one
+// warp per canonical list split (S, a context property).  KP changes only how the items are cut into warps --
+// never a result (vs_cells.cu header) -- so it is chosen per launch for speed: KP 2 unless the run's scoring round
+// (all its spots) would have fewer than fill_warps warps, then KP 1 (twice the warps, each with half the items) for
+// latency-bound launches (few spots, Improve's m poses per spot).  (A warp looping over several splits was
+// measured slower than one warp per split even for latency-bound launches: profiles/r02_notes.md.)
+struct Shape {
+  int kp, H, cn, chb, w, S;
+  int nsg() const { return S; }
+};
+Shape shape_of(const vs_ctx* c, int kp, int w) {
+  Shape s;
+  s.S = c->nsplit;
+  s.kp = kp;
+  s.H = kp == 2 ? c->H2 : c->H1;
+  s.cn = 64 * kp;
+  s.chb = 64 * s.H;
+  s.w = w;
+  return s;
+}
+Shape choose_shape(const vs_ctx* c, long long n_seg, int seg_n) {
+  if (c->force_kp) return shape_of(c, c->force_kp, 1);
+  const Shape s2 = shape_of(c, 2, 1);
+  if (n_seg * cell_chunks(seg_n, c->nn, c->nh, s2.cn, s2.chb) * s2.nsg() >= c->fill_warps) return s2;
+  return shape_of(c, 1, 1);
+}
+void apply_shape(CellArgs& a, const Shape& s) {
+  a.kp = s.kp;
+  a.H = s.H;
+  a.cn = s.cn;
+  a.chb = s.chb;
+  a.w = s.w;
+  a.nsplit = s.S;
 }
 
 CellArgs cell_base(vs_ctx* c) {
@@ -339,14 +376,11 @@ CellArgs cell_base(vs_ctx* c) {
   a.n_lig = c->n_lig;
   a.nn = c->nn;
   a.nh = c->nh;
-  a.H = c->H;
-  a.cn = c->cn;
-  a.chb = c->chb;
+  apply_shape(a, shape_of(c, 2, 4));
   a.shift = c->d_shift;
   a.W = c->W;
   a.inv_hm = c->inv_hm;
   a.cut = c->all_pairs ? 0 : 1;
-  a.nsplit = 1;
   a.K = 1;
   a.r2min = c->r2min;
   a.rc = c->rc;
@@ -356,11 +390,17 @@ CellArgs cell_base(vs_ctx* c) {
   a.hbD = c->hbD;
   a.T = c->T;
   a.counters = c->d_counters;
+  a.census = c->census ? 1 : 0;
+  a.kt = c->ktime ? c->d_kt : nullptr;
+  a.kt_base = c->d_kt_base;
+  a.kt_cap = VS_KT_CAP;
   a.seedp = c->d_seed;
   return a;
 }
 
-vs_status cell_launch(vs_ctx* c, const CellArgs& a, long long n_poses, int nb2, cudaStream_t st) {
+vs_status cell_launch(vs_ctx* c, const CellArgs& a_in, long long n_poses, int nb2, cudaStream_t st) {
+  CellArgs a = a_in;
+  if (a.kt) a.kt_slot = c->kt_local++;
   cudaEvent_t e0 = nullptr, e1 = nullptr;
   const bool timed = c->timing && !c->capturing;
   if (timed) {
@@ -421,7 +461,8 @@ struct Body {
   PoseRec* pbuf;
   float4* items;
   double* E;
-  int emax;  // E entries per spot and ligand atom: max over the launches of (poses per spot x list splits)
+  int emax;  // E entries per spot and ligand atom: max over the launches of (poses per spot x split groups)
+  int census, ktime;  // instrumentation (a different pair-kernel instantiation / extra arguments)
 };
 
 static_assert(sizeof(Body) <= 256, "graph key storage");
@@ -504,6 +545,7 @@ vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, int g, Tr
 vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
   const vs_mh_params* mp = &b.mp;
   const int P = mp->population, m = b.m, ns = b.ns;
+  c->kt_local = 0;
   // Spots are independent: split them into groups whose generation loops run on separate
   // streams, enqueued generation by generation, so one group's kernels fill the wave tails of
   // another's.
@@ -529,8 +571,10 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     if (G > 1) CK(cudaStreamWaitEvent(q.st, c->ev_fork, 0), "stream wait");
     {
       const int mk = m * mp->ls_neighbours, maxpose = std::max(P, mk);
+      const Shape shp = choose_shape(c, ns, P), shl = choose_shape(c, ns, mk);  // shapes from the whole run's size
       CellArgs& cp = q.cplain;
       cp = cell_base(c);
+      apply_shape(cp, shp);
       cp.nseg = q.ns;
       cp.seg_spot = q.seg;
       cp.uniform = 1;
@@ -538,26 +582,25 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
       cp.seg_stride = P;
       cp.P = P;
       cp.mode = MODE_PLAIN;
-      cp.nch_u = cell_chunks(P, c->nn, c->nh, c->cn, c->chb);
-      cp.nsplit = cell_nsplit(cp.nch_u, c->split_warps);
+      cp.nch_u = cell_chunks(P, c->nn, c->nh, shp.cn, shp.chb);
       cp.pbuf = b.pbuf + (size_t)k0 * maxpose;
       cp.items = b.items + (size_t)k0 * maxpose * c->n_lig;
       cp.E = b.E + (size_t)k0 * c->n_lig * b.emax;
       cp.E_stride = (long long)q.ns * P * c->n_lig;
       CellArgs& cl = q.cls;
       cl = cp;
+      apply_shape(cl, shl);
       cl.mode = MODE_LS;
       cl.seg_size = mk;
-      cl.nch_u = cell_chunks(mk, c->nn, c->nh, c->cn, c->chb);
-      cl.nsplit = cell_nsplit(cl.nch_u, c->split_warps);
+      cl.nch_u = cell_chunks(mk, c->nn, c->nh, shl.cn, shl.chb);
       cl.E_stride = (long long)q.ns * mk * c->n_lig;
       cl.J = q.J;
       cl.m = m;
       cl.K = mp->ls_neighbours;
       cl.ls_trans = mp->ls_trans;
       cl.ls_rot = mp->ls_rot;
-      q.cplain_blocks = q.ns * cp.nch_u * cp.nsplit;
-      q.cls_blocks = q.ns * cl.nch_u * cl.nsplit;
+      q.cplain_blocks = q.ns * cp.nch_u * shp.nsg();
+      q.cls_blocks = q.ns * cl.nch_u * shl.nsg();
     }
   }
   vs_status r;
@@ -573,6 +616,10 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
     }
   CK(launch_best(grp[0].in_b ? b.SB : b.SA, ns, P, b.best_pose, b.best_score, st), "best launch");
   c->launches++;
+  if (b.ktime) {
+    CK(launch_kt_advance(c->d_kt_base, c->kt_local, st), "kt launch");
+    c->launches++;
+  }
   return VS_OK;
 }
 
@@ -602,8 +649,8 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     const int mk = m * mp->ls_neighbours, maxpose = std::max(P, mk);
     if ((long long)ns * maxpose * c->n_lig >= (1ll << 31))
       return set_err(VS_ERR_INVALID_ARGUMENT, "n_sel x population x n_lig must be < 2^31");
-    emax = P * cell_nsplit(cell_chunks(P, c->nn, c->nh, c->cn, c->chb), c->split_warps);
-    if (mp->improve_frac > 0.0f) emax = std::max(emax, mk * cell_nsplit(cell_chunks(mk, c->nn, c->nh, c->cn, c->chb), c->split_warps));
+    emax = P * choose_shape(c, ns, P).nsg();
+    if (mp->improve_frac > 0.0f) emax = std::max(emax, mk * choose_shape(c, ns, mk).nsg());
     CK(c->buf[B_PBUF].ensure(sizeof(PoseRec) * (size_t)ns * maxpose), "alloc");
     CK(c->buf[B_ITEMS].ensure(sizeof(float4) * (size_t)ns * maxpose * c->n_lig), "alloc");
     CK(c->buf[B_E].ensure(sizeof(double) * (size_t)ns * c->n_lig * emax), "alloc");
@@ -633,24 +680,30 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     b.E = (double*)c->buf[B_E].p;
     b.emax = emax;
   }
+  b.census = c->census ? 1 : 0;
+  b.ktime = c->ktime ? 1 : 0;
   if (tr || !c->graphs) return enqueue_body(c, b, st, tr);
 
   // CUDA graph of the whole run: captured on the second identical call, replayed afterwards
   // (the ~4 + 2 L launches per generation and spot group then cost one graph launch).
-  const bool same_as_cached = c->gexec && std::memcmp(&b, &c->gkey, sizeof(Body)) == 0;
-  if (same_as_cached) {
-    CK(cudaGraphLaunch(c->gexec, st), "graph launch");
-    c->launches += c->g_launches;
-    c->score_launches += c->g_score_launches;
-    return VS_OK;
-  }
+  for (auto& gr : c->gcache)
+    if (std::memcmp(&b, gr.key, sizeof(Body)) == 0) {
+      CK(cudaGraphLaunch(gr.exec, st), "graph launch");
+      c->launches += gr.launches;
+      c->score_launches += gr.score_launches;
+      gr.used = ++c->gclock;
+      return VS_OK;
+    }
   const bool seen = c->has_last && std::memcmp(&b, &c->last_key, sizeof(Body)) == 0;
   std::memcpy(&c->last_key, &b, sizeof(Body));
   c->has_last = true;
   if (!seen) return enqueue_body(c, b, st, tr);
-  if (c->gexec) {
-    cudaGraphExecDestroy(c->gexec);
-    c->gexec = nullptr;
+  if (c->gcache.size() >= VS_GRAPH_CACHE) {  // evict the least recently used graph
+    size_t lru = 0;
+    for (size_t i = 1; i < c->gcache.size(); ++i)
+      if (c->gcache[i].used < c->gcache[lru].used) lru = i;
+    cudaGraphExecDestroy(c->gcache[lru].exec);
+    c->gcache.erase(c->gcache.begin() + lru);
   }
   const uint64_t l0 = c->launches, s0 = c->score_launches;
   CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal), "begin capture");
@@ -664,13 +717,16 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     return r;
   }
   CK(e, "end capture");
-  e = cudaGraphInstantiate(&c->gexec, graph, 0);
+  vs_ctx::Graph gr;
+  e = cudaGraphInstantiate(&gr.exec, graph, 0);
   cudaGraphDestroy(graph);
   CK(e, "graph instantiate");
-  std::memcpy(&c->gkey, &b, sizeof(Body));
-  c->g_launches = c->launches - l0;
-  c->g_score_launches = c->score_launches - s0;
-  CK(cudaGraphLaunch(c->gexec, st), "graph launch");
+  std::memcpy(gr.key, &b, sizeof(Body));
+  gr.launches = c->launches - l0;
+  gr.score_launches = c->score_launches - s0;
+  gr.used = ++c->gclock;
+  c->gcache.push_back(gr);
+  CK(cudaGraphLaunch(gr.exec, st), "graph launch");
   return VS_OK;
 }
 
@@ -679,8 +735,11 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
                              float* d_out, cudaStream_t st) {
   const int ns = c->n_spots;
   const int64_t slice = std::max<int64_t>(1, (int64_t(1) << 26) / c->n_lig);
+  c->kt_local = 0;
   for (int64_t o = 0; o < n; o += slice) {
     const int64_t nb = std::min(slice, n - o);
+    // launch shape from the slice's size (poses spread over the spots: one segment of nb poses approximates it)
+    const Shape sh = choose_shape(c, 1, (int)nb);
     const int32_t* sp = d_spot + o;
     const float* q = d_q + 4 * o;
     const float* t = d_t + 3 * o;
@@ -694,7 +753,7 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
     CK(c->buf[B_ORIG].ensure(sizeof(int) * nb), "alloc");
     CK(c->buf[B_PBUF].ensure(sizeof(PoseRec) * nb), "alloc");
     CK(c->buf[B_ITEMS].ensure(sizeof(float4) * nb * c->n_lig), "alloc");
-    CK(c->buf[B_E].ensure(sizeof(double) * nb * c->n_lig), "alloc");
+    CK(c->buf[B_E].ensure(sizeof(double) * nb * c->n_lig * sh.nsg()), "alloc");
     int* valid = (int*)c->buf[B_VALID].p;
     int* counts = (int*)c->buf[B_COUNTS].p;
     int* pp = (int*)c->buf[B_PP].p;
@@ -704,10 +763,11 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
     int* orig = (int*)c->buf[B_ORIG].p;
     CK(cudaMemsetAsync(counts, 0, sizeof(int) * ns, st), "memset");
     CK(launch_validate(nb, sp, q, t, ns, c->T, c->all_pairs ? 0 : 1, valid, counts, out, st), "validate launch");
-    CK(launch_cell_scan(counts, ns, c->nn, c->nh, c->cn, c->chb, pp, cp, cur, st), "scan launch");
+    CK(launch_cell_scan(counts, ns, c->nn, c->nh, sh.cn, sh.chb, pp, cp, cur, st), "scan launch");
     CK(launch_scatter(nb, sp, q, t, valid, cur, sorted, orig, st), "scatter launch");
     c->launches += 3;
     CellArgs a = cell_base(c);
+    apply_shape(a, sh);
     a.nseg = ns;
     a.seg_spot = c->d_iota;
     a.uniform = 0;
@@ -722,12 +782,38 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
     a.E = (double*)c->buf[B_E].p;
     a.E_stride = nb * c->n_lig;
     // pair-kernel grid: an upper bound of sum_k cell_chunks(n_k) (<= n_k n_lig / cn + n_k nh / chb + 3)
-    int64_t blocks = 3 * (int64_t)ns + (nb * c->n_lig) / c->cn + 1;
-    if (c->chb > 0) blocks += (nb * c->nh) / c->chb;
+    int64_t blocks = 3 * (int64_t)ns + (nb * c->n_lig) / sh.cn + 1;
+    if (sh.chb > 0) blocks += (nb * c->nh) / sh.chb;
+    blocks *= sh.nsg();
     if (blocks > 0x7fffffff) return set_err(VS_ERR_INVALID_ARGUMENT, "too many poses in one call");
     vs_status r = cell_launch(c, a, nb, (int)blocks, st);
     if (r != VS_OK) return r;
   }
+  if (c->ktime) {
+    CK(launch_kt_advance(c->d_kt_base, c->kt_local, st), "kt launch");
+    c->launches++;
+  }
+  return VS_OK;
+}
+
+// The asynchronous entry points run on the ctx's own stream, ordered after the caller's stream and before its
+// later work by an event pair: the ctx's scratch buffers are then used by one stream only (no overlap between a
+// vs_score_poses_device and a vs_run_async of the same ctx), and graph capture always happens on a capturable
+// (non-legacy) stream whatever the caller passes (NULL = the legacy default stream included).
+vs_status join_in(vs_ctx* c, cudaStream_t caller) {
+#ifdef VS_NO_JOIN
+  return VS_OK;
+#endif
+  CK(cudaEventRecord(c->ev_in, caller), "event record (caller stream)");
+  CK(cudaStreamWaitEvent(c->stream, c->ev_in, 0), "stream wait");
+  return VS_OK;
+}
+vs_status join_out(vs_ctx* c, cudaStream_t caller) {
+#ifdef VS_NO_JOIN
+  return VS_OK;
+#endif
+  CK(cudaEventRecord(c->ev_out, c->stream), "event record");
+  CK(cudaStreamWaitEvent(caller, c->ev_out, 0), "stream wait (caller stream)");
   return VS_OK;
 }
 
@@ -755,6 +841,7 @@ void vs_score_params_default(vs_score_params* o) {
   o->type_sigma = nullptr;
   o->type_eps = nullptr;
   o->type_hb_role = nullptr;
+  o->list_splits = 0;
 }
 
 vs_status vs_mh_preset(int m, vs_mh_params* o) {
@@ -791,6 +878,10 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
       !(sp.hb_eps >= 0.0f && std::isfinite(sp.hb_eps)) || !(sp.hb_r0 > 0.0f && std::isfinite(sp.hb_r0)) ||
       !(sp.r2_min > 0.0f && std::isfinite(sp.r2_min)) || std::isnan(sp.cutoff))
     return set_err(VS_ERR_INVALID_ARGUMENT, "invalid score params");
+  // list_splits 0 = by the context's spot count: few spots -> latency-bound runs -> more splits (R32)
+  if (sp.list_splits == 0) sp.list_splits = n_spots <= 128 ? 4 : (n_spots <= 256 ? 2 : 1);
+  if (sp.list_splits != 1 && sp.list_splits != 2 && sp.list_splits != 4)
+    return set_err(VS_ERR_INVALID_ARGUMENT, "list_splits must be 0, 1, 2 or 4");
   if (sp.n_types < 0 || sp.n_types > 64 || (sp.n_types > 0 && (!sp.type_sigma || !sp.type_eps || !sp.type_hb_role)))
     return set_err(VS_ERR_INVALID_ARGUMENT, "invalid type table");
   if (!finite_arr(rec_xyz, 3 * (int64_t)n_rec) || !finite_arr(rec_q, n_rec) || !finite_arr(lig_xyz, 3 * (int64_t)n_lig) ||
@@ -833,9 +924,15 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   c->n_rec = n_rec;
   c->n_lig = n_lig;
   c->n_spots = n_spots;
-  c->split_warps = std::max(VS_SPLIT_WARPS, std::min(VS_SPLIT_WARPS_MAX, VS_SPLIT_TOTAL / std::max(1, (int)n_spots)));
+  // launch-shape knobs for experiments (speed only; results never depend on them)
+  if (const char* v = std::getenv("VS_FILL_WARPS")) c->fill_warps = std::max(1ll, std::atoll(v));
+  if (const char* v = std::getenv("VS_SHAPE")) {  // "kp"
+    const int kp = std::atoi(v);
+    if (kp == 1 || kp == 2) c->force_kp = kp;
+  }
   c->all_pairs = !(sp.cutoff > 0.0f) || std::isinf(sp.cutoff);
   c->dielectric = sp.dielectric;
+  c->nsplit = sp.list_splits;
   c->T = sp.region_half_width;
   c->rc = c->all_pairs ? INFINITY : sp.cutoff;
   c->rc2 = c->all_pairs ? INFINITY : (float)((double)sp.cutoff * sp.cutoff);
@@ -860,6 +957,8 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     CKC(cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming), "event create");
   }
   CKC(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming), "event create");
+  CKC(cudaEventCreateWithFlags(&c->ev_in, cudaEventDisableTiming), "event create");
+  CKC(cudaEventCreateWithFlags(&c->ev_out, cudaEventDisableTiming), "event create");
   // ligand: centred on the fp32-rounded fp64 centroid (R11)
   float cen[3];
   for (int a = 0; a < 3; ++a) {
@@ -898,9 +997,10 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     }
     c->nn = cnt[0];
     c->nh = cnt[1];
-    // H-bond slot pairs per lane: the launch-uniform H minimising (chunks per pose) x (issue slots per chunk),
-    // with 19 slots per class-0-only pair and 23 per H-bond pair; class-0 items may overflow
-    // into H-bond slots, so chunks per pose = max(n / CH_ITEMS, nh / (64 H))
+    // H-bond slot pairs per lane of the KP = 2 kernel: the H minimising (chunks per pose) x (issue slots per
+    // chunk), with 19 slots per class-0-only pair and 23 per H-bond pair; class-0 items may
+    // overflow into H-bond slots, so chunks per pose = max(n / CH_ITEMS, nh / (64 H)).  The KP = 1 kernel has
+    // one slot pair: an H-bond pair whenever the ligand has H-bond atoms.
     double best = 1e300;
     for (int h = merge ? CELL_KP : 0; h <= CELL_KP; ++h) {
       if (c->nh > 0 && h == 0) continue;
@@ -908,11 +1008,10 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
       const double cost = per * (19.0 * (CELL_KP - h) + 23.0 * h);
       if (cost < best - 1e-12) {
         best = cost;
-        c->H = h;
+        c->H2 = h;
       }
     }
-    c->cn = CH_ITEMS;
-    c->chb = 64 * c->H;
+    c->H1 = c->nh > 0 ? 1 : 0;
     CKC(pool::alloc(&c->d_ligx, sizeof(float4) * n_lig), "alloc ligand");
     CKC(pool::alloc(&c->d_ligp, sizeof(float4) * n_lig), "alloc ligand");
     CKC(pool::alloc(&c->d_lig_rank, sizeof(int) * n_lig), "alloc ligand");
@@ -1019,13 +1118,13 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   CKT(cudaMemcpyAsync(c->d_shift, h_shift.data(), sizeof(float4) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
   CKT(pool::alloc(&c->d_iota, sizeof(int) * n_spots), "alloc");
   CKT(cudaMemcpyAsync(c->d_iota, iota.data(), sizeof(int) * n_spots, cudaMemcpyHostToDevice, c->stream), "H2D");
-  CKT(pool::alloc(&c->d_counters, sizeof(unsigned long long) * 3), "alloc");
+  CKT(pool::alloc(&c->d_counters, sizeof(unsigned long long) * 4), "alloc");
   CKT(pool::alloc(&c->d_seed, sizeof(uint64_t)), "alloc");
   {
     const char* gv = std::getenv("VS_GRAPHS");
     c->graphs = !(gv && gv[0] == '0');
   }
-  CKT(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 3), "memset");
+  CKT(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 4), "memset");
   CKT(cudaStreamSynchronize(c->stream), "sync");
   free_tmp();
   c->h_list_len = h_len;
@@ -1076,7 +1175,10 @@ vs_status vs_score_poses_device(vs_ctx* c, int64_t n, const int32_t* d_spot, con
   if (n == 0) return VS_OK;
   if (!d_spot || !d_q || !d_t || !d_score) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL pose array");
   DeviceGuard guard(c->dev);
-  return score_device_impl(c, n, d_spot, d_q, d_t, d_score, (cudaStream_t)stream);
+  vs_status r = join_in(c, (cudaStream_t)stream);
+  if (r == VS_OK) r = score_device_impl(c, n, d_spot, d_q, d_t, d_score, c->stream);
+  if (r == VS_OK) r = join_out(c, (cudaStream_t)stream);
+  return r;
 }
 
 static vs_status run_host(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_sel, const int32_t* spot_ids,
@@ -1117,7 +1219,14 @@ vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t
   if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
   if (!d_best_pose || !d_best_score) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL output");
   DeviceGuard guard(c->dev);
-  return run_impl(c, mp, seed, n_sel, spot_ids, d_best_pose, d_best_score, (cudaStream_t)stream, nullptr);
+  vs_status r = join_in(c, (cudaStream_t)stream);
+#ifdef VS_NO_JOIN
+  if (r == VS_OK) r = run_impl(c, mp, seed, n_sel, spot_ids, d_best_pose, d_best_score, (cudaStream_t)stream, nullptr);
+#else
+  if (r == VS_OK) r = run_impl(c, mp, seed, n_sel, spot_ids, d_best_pose, d_best_score, c->stream, nullptr);
+#endif
+  if (r == VS_OK) r = join_out(c, (cudaStream_t)stream);
+  return r;
 }
 
 // VS_DEBUG_TIMING=1: phase times of vs_destroy on stderr (host-side cost investigation)
@@ -1143,10 +1252,10 @@ void vs_destroy(vs_ctx* c) {
   for (auto& b : c->buf) b.release();
   lap(1);
   for (auto e : c->ev) cudaEventDestroy(e);
-  if (c->gexec) cudaGraphExecDestroy(c->gexec);
+  for (auto& gr : c->gcache) cudaGraphExecDestroy(gr.exec);
   lap(2);
   void* ptrs[] = {c->d_lists, c->d_list_off, c->d_list_len, c->d_shift, c->d_iota, c->d_counters,
-                  c->d_seed, c->d_cells, c->d_ligx, c->d_ligp, c->d_lig_rank};
+                  c->d_seed, c->d_cells, c->d_ligx, c->d_ligp, c->d_lig_rank, c->d_kt, c->d_kt_base};
   for (void* p : ptrs)
     if (p) pool::release(p);
   lap(3);
@@ -1156,6 +1265,8 @@ void vs_destroy(vs_ctx* c) {
     if (c->ev_join[i]) cudaEventDestroy(c->ev_join[i]);
   }
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_in) cudaEventDestroy(c->ev_in);
+  if (c->ev_out) cudaEventDestroy(c->ev_out);
   lap(4);
   delete c;
   if (debug_timing())
@@ -1183,9 +1294,20 @@ vs_status vs_release_cached_memory(int32_t cuda_device) {
 const char* vs_last_error(void) { return g_err.c_str(); }
 int vs_abi_version(void) { return VS_ABI_VERSION; }
 
-vs_status vs_set_timing(vs_ctx* c, int enable) {
+vs_status vs_set_timing(vs_ctx* c, int flags) {
   if (!c) return set_err(VS_ERR_INVALID_ARGUMENT, "ctx: NULL");
-  c->timing = enable != 0;
+  if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
+  DeviceGuard guard(c->dev);
+  if ((flags & VS_TIMING_KERNEL) && !c->d_kt) {
+    CK(cudaStreamSynchronize(c->stream), "sync");
+    CK(pool::alloc(&c->d_kt, sizeof(unsigned long long) * 2 * (size_t)VS_KT_CAP), "alloc");
+    CK(pool::alloc(&c->d_kt_base, sizeof(unsigned long long)), "alloc");
+    CK(cudaMemset(c->d_kt, 0, sizeof(unsigned long long) * 2 * (size_t)VS_KT_CAP), "memset");
+    CK(cudaMemset(c->d_kt_base, 0, sizeof(unsigned long long)), "memset");
+  }
+  c->timing = (flags & VS_TIMING_EVENTS) != 0;
+  c->ktime = (flags & VS_TIMING_KERNEL) != 0;
+  c->census = (flags & VS_TIMING_CENSUS) != 0;
   return VS_OK;
 }
 
@@ -1196,8 +1318,41 @@ vs_status vs_get_stats(vs_ctx* c, vs_stats* o) {
   CK(cudaDeviceSynchronize(), "sync");
   vs_status s = collect_timing(c);
   if (s != VS_OK) return s;
-  unsigned long long h[3];
+  unsigned long long h[4];
   CK(cudaMemcpy(h, c->d_counters, sizeof(h), cudaMemcpyDeviceToHost), "D2H counters");
+  o->pairs_within = c->all_pairs ? h[2] : h[3];  // all-pairs mode: every pair is within
+  o->pair_busy_ms = o->pair_launch_ms = 0.0;
+  o->pair_timed_launches = 0;
+  if (c->d_kt) {  // pair-kernel launch intervals: their sum and the length of their union
+    unsigned long long nslot = 0;
+    CK(cudaMemcpy(&nslot, c->d_kt_base, sizeof(nslot), cudaMemcpyDeviceToHost), "D2H kt");
+    nslot = std::min<unsigned long long>(nslot, VS_KT_CAP);
+    std::vector<unsigned long long> kt(2 * nslot);
+    if (nslot) CK(cudaMemcpy(kt.data(), c->d_kt, sizeof(unsigned long long) * 2 * nslot, cudaMemcpyDeviceToHost), "D2H kt");
+    std::vector<std::pair<unsigned long long, unsigned long long>> iv;
+    for (unsigned long long i = 0; i < nslot; ++i)
+      if (kt[2 * i] && kt[2 * i + 1]) iv.emplace_back(~kt[2 * i], kt[2 * i + 1]);
+    std::sort(iv.begin(), iv.end());
+    double sum = 0.0, busy = 0.0;
+    unsigned long long cs = 0, ce = 0;
+    bool open = false;
+    for (auto& x : iv) {
+      if (x.second < x.first) continue;
+      sum += (double)(x.second - x.first);
+      if (!open || x.first > ce) {
+        if (open) busy += (double)(ce - cs);
+        cs = x.first;
+        ce = x.second;
+        open = true;
+      } else if (x.second > ce) {
+        ce = x.second;
+      }
+    }
+    if (open) busy += (double)(ce - cs);
+    o->pair_busy_ms = busy * 1e-6;
+    o->pair_launch_ms = sum * 1e-6;
+    o->pair_timed_launches = iv.size();
+  }
   o->kernel_launches = c->launches;
   o->score_launches = c->score_launches;
   o->pairs = h[2];
@@ -1213,7 +1368,11 @@ vs_status vs_reset_stats(vs_ctx* c) {
   if (c->poisoned) return set_err(VS_ERR_CUDA, "ctx poisoned by an earlier CUDA error");
   DeviceGuard guard(c->dev);
   CK(cudaDeviceSynchronize(), "sync");
-  CK(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 3), "memset");
+  CK(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 4), "memset");
+  if (c->d_kt) {
+    CK(cudaMemset(c->d_kt, 0, sizeof(unsigned long long) * 2 * (size_t)VS_KT_CAP), "memset");
+    CK(cudaMemset(c->d_kt_base, 0, sizeof(unsigned long long)), "memset");
+  }
   c->ev_used = 0;
   c->launches = c->score_launches = 0;
   c->score_ms_acc = 0.0;

@@ -68,11 +68,9 @@ enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
 constexpr int CELL_G = VS_CELL_G;                  // list grid per spot: G^3 cells over [-R, R]^3 (G <= 64)
 constexpr int CELL_G3 = CELL_G * CELL_G * CELL_G;
 constexpr int CELL_SORT_MAX = 16384;               // longest list cell-sorted in shared memory (128 KB keys)
-#ifndef VS_CELL_KP
-#define VS_CELL_KP 2
-#endif
-constexpr int CELL_KP = VS_CELL_KP;                // packed float2 item pairs per lane (register blocking)
-constexpr int CH_ITEMS = 2 * CELL_KP * 32;         // items per chunk (one warp)
+constexpr int CELL_KP = 2;                         // packed float2 item pairs per lane of the default pair kernel
+constexpr int CH_ITEMS = 2 * CELL_KP * 32;         // items per chunk (one warp) of the default pair kernel
+constexpr int CELL_NSPLIT = 4;                     // most canonical receptor-list splits (item energy (e0+e1)+(e2+e3))
 #ifndef VS_CELL_BATCH
 #define VS_CELL_BATCH 64
 #endif
@@ -94,8 +92,11 @@ struct CellArgs {
   const float4* ligp;        // es_i, c12_i, c6_i, donor_i
   const int* lig_rank;       // rank of the atom within its class
   int n_lig, nn, nh;         // atoms, of which nn without / nh with an H-bond role
-  int H;                     // H-bond slot pairs per lane (launch-uniform; the first CELL_KP - H pairs hold class 0 only)
-  int cn, chb;               // chunk capacities: cn = CH_ITEMS items in all, chb = 64 H class-1 items
+  // launch shape (speed only, never results): kp packed item pairs per lane (1 or 2), H of them H-bond pairs (the
+  // first kp - H pairs hold class 0 only), chunk capacities cn = 64 kp items, chb = 64 H class-1 items (w: 1)
+  int kp, H, cn, chb, w;
+  int nsplit;                // canonical list splits S (1, 2, 4) of the context, one warp each: the split tree
+                             // (e0 + e1) + (e2 + e3) of an item's split energies defines the result
   const float4* shift;       // added to t + R l (all-pairs: 0 -- lists are spot-relative)
   float W, inv_hm;           // item sort grid: [-W, W]^3, 16 cells per axis
   int cut;                   // cutoff mode (cell culling, spatial item sort)
@@ -106,7 +107,6 @@ struct CellArgs {
   const int* pose_prefix;    // non-uniform: [nseg + 1]
   const int* chunk_prefix;   // non-uniform: [nseg + 1]
   int nch_u;                 // uniform: chunks per segment
-  int nsplit;                // list splits per chunk (partial energies summed by the finalize kernel)
   // poses
   int mode;                  // MODE_PLAIN / MODE_LS
   PoseRec* poses;            // PLAIN: segment k pose p at k * seg_stride + p (uniform) or pose_prefix[k] + p;
@@ -122,11 +122,16 @@ struct CellArgs {
   // launch scratch
   PoseRec* pbuf;             // [launch poses] the pose scored (LS: the proposal, t.w = score of X[j])
   float4* items;             // [launch items] per segment: class-0 items then class-1 items, each spatially sorted
-  double* E;                 // [nsplit][launch items] per-item energies
+  double* E;                 // [nsplit][launch items] per-item energies of each split
   long long E_stride;
   float r2min, rc, rc2, inv_rc2;
   float hbC, hbD;
-  unsigned long long* counters;  // [0] pairs evaluated, [1] poses, [2] workload pairs
+  unsigned long long* counters;  // [0] pairs evaluated, [1] poses, [2] workload pairs, [3] pairs within rc (census)
+  int census;                // count the pairs within rc (a separate pair-kernel instantiation; same results)
+  // instrumentation: pair-kernel launch intervals (globaltimer) in slot kt_slot of the run's region at *kt_base
+  unsigned long long* kt;
+  const unsigned long long* kt_base;
+  int kt_slot, kt_cap;
 };
 
 // Chunks of a segment of seg_n poses: class-1 items (H-bond role) fill at most cap1 = 64 H slots (the last H
@@ -145,6 +150,7 @@ cudaError_t launch_cell_sort(const RecAtom* lists, RecAtom* out, const int* off,
                              float R, float inv_h, cudaStream_t st);
 // K1 + K2 + K3 of one scoring call; n_blocks2 = pair-kernel grid (upper bound when non-uniform)
 cudaError_t launch_cell_score(const CellArgs& a, int dielectric, long long n_poses, int n_blocks2, cudaStream_t st);
+cudaError_t launch_kt_advance(unsigned long long* kt_base, int slots, cudaStream_t st);
 cudaError_t launch_cell_scan(const int* counts, int n, int nn, int nh, int cn, int chb, int* pose_prefix,
                              int* chunk_prefix, int* cursor, cudaStream_t st);
 

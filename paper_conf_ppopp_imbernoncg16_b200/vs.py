@@ -16,6 +16,7 @@ import numpy as np
 from . import build as _build
 
 OK, ERR_INVALID_ARGUMENT, ERR_POSE_OUT_OF_REGION, ERR_ZERO_QUATERNION, ERR_CUDA, ERR_OUT_OF_MEMORY, ERR_UNSUPPORTED = range(7)
+TIMING_EVENTS, TIMING_KERNEL, TIMING_CENSUS = 1, 2, 4   # vs_set_timing flags (include/vs.h)
 TRACE_INIT, TRACE_SCORED, TRACE_SELECT, TRACE_LS, TRACE_SORTED, TRACE_COMBINED, TRACE_INCLUDED = range(7)
 
 # every symbol include/vs.h declares (checked by tests/test_abi.py)
@@ -43,7 +44,8 @@ class ScoreParams(C.Structure):
     _fields_ = [("coulomb_k", C.c_float), ("dielectric", C.c_int), ("eps_r", C.c_float), ("cutoff", C.c_float),
                 ("region_half_width", C.c_float), ("hb_eps", C.c_float), ("hb_r0", C.c_float),
                 ("r2_min", C.c_float), ("n_types", C.c_int), ("type_sigma", C.POINTER(C.c_float)),
-                ("type_eps", C.POINTER(C.c_float)), ("type_hb_role", C.POINTER(C.c_int))]
+                ("type_eps", C.POINTER(C.c_float)), ("type_hb_role", C.POINTER(C.c_int)),
+                ("list_splits", C.c_int)]
 
 
 class MHParams(C.Structure):
@@ -56,7 +58,8 @@ class MHParams(C.Structure):
 class Stats(C.Structure):
     _fields_ = [("kernel_launches", C.c_uint64), ("score_launches", C.c_uint64), ("poses_scored", C.c_uint64),
                 ("pairs", C.c_uint64), ("score_ms", C.c_double), ("timed_launches", C.c_uint64),
-                ("pairs_evaluated", C.c_uint64)]
+                ("pairs_evaluated", C.c_uint64), ("pairs_within", C.c_uint64), ("pair_busy_ms", C.c_double),
+                ("pair_launch_ms", C.c_double), ("pair_timed_launches", C.c_uint64)]
 
     def asdict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -254,8 +257,10 @@ class Context:
         return pose, sc
 
     # ---- instrumentation
-    def set_timing(self, enable: bool = True):
-        _check(load().vs_set_timing(self.h, 1 if enable else 0))
+    def set_timing(self, enable=True):
+        """enable: bool (CUDA events around un-graphed scoring calls) or an OR of TIMING_* flags."""
+        flags = int(enable) if not isinstance(enable, bool) else (TIMING_EVENTS if enable else 0)
+        _check(load().vs_set_timing(self.h, flags))
 
     def stats(self) -> dict:
         s = Stats()

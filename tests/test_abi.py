@@ -24,7 +24,7 @@ def test_library_exports_every_declared_symbol():
     L = vs.load()
     for name in declared_symbols():
         assert hasattr(L, name), name
-    assert L.vs_abi_version() == 3
+    assert L.vs_abi_version() == 4
 
 
 def test_library_targets_sm100a():

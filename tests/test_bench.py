@@ -25,6 +25,8 @@ def test_reference_arm_line():
     d = _run([sys.executable, "bench.py", "--impl", "reference", "--config", "tiny", "--steps", "1", "--warmup", "0"])
     assert d["impl"] == "reference" and d["value"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
     assert d["e2e"]["h2d_bytes_per_step"] == 0
+    # value counts the pairs within rc, the oracle visits every receptor atom
+    assert d["value"] <= d["workload_pairs_per_s"] <= d["visited_pairs_per_s"]
 
 
 @pytest.mark.gpu
@@ -32,20 +34,30 @@ def test_bench_single_gpu_line():
     d = _run([sys.executable, "bench.py", "--config", "small", "--steps", "2", "--warmup", "3", "--generations", "4"])
     assert KEYS <= set(d)
     assert d["n_gpus"] == 1 and d["value"] > 0 and d["gpu_launches"] > 0
+    assert d["value"] < d["pairs_evaluated_per_s"] < d["workload_pairs_per_s"]
     r = d["roofline"]
-    assert r["bound"] == "alu" and 0 < r["frac"] < 3 and r["peak"] > 0
+    assert r["bound"] == "alu" and 0 < r["frac"] < 1.5 and r["peak"] > 0
+    assert 0 < r["pair_kernel_share_of_step"] <= 1.05 and r["pair_kernel_launches"] > 0
+    assert d["check"]["assembled_equals_single_process"] is True
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["cpu_baseline"]["cores"] >= 1
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("scaling", ["weak", "strong"])
-def test_bench_two_ranks_gloo_on_one_gpu(scaling):
-    """The torchrun path (queue, gather, max-over-ranks timing) with gloo collectives on one GPU."""
-    d = _run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
-              "--master-addr", "127.0.0.1", "--master-port", "29517" if scaling == "weak" else "29519",
-              "bench.py", "--gpus", "2", "--config", "small", "--steps", "1", "--warmup", "3", "--generations", "3",
-              "--scaling", scaling, "--no-micro", "--no-cpu-baseline"], env={"VS_BENCH_BACKEND": "gloo"})
-    assert d["n_gpus"] == 2 and d["scaling"] == scaling and d["value"] > 0
+@pytest.mark.parametrize("extra", [["--scaling", "replicas"], ["--schedule", "queue", "--chunks-per-rank", "3",
+                                                                "--slots", "2"],
+                                   ["--schedule", "warmup", "--hetero", "0:2"], ["--schedule", "static"]])
+def test_bench_two_ranks_gloo_on_one_gpu(extra):
+    """--gpus 2 re-launches itself under torch.distributed.run; gloo collectives let both ranks share one GPU.
+    The gathered, assembled per-spot bests must equal a single-process run bit for bit."""
+    d = _run([sys.executable, "bench.py", "--gpus", "2", "--config", "small", "--steps", "1", "--warmup", "3",
+              "--generations", "3", "--no-micro", "--no-cpu-baseline"] + extra, env={"VS_BENCH_BACKEND": "gloo"})
+    assert d["n_gpus"] == 2 and d["value"] > 0
+    assert all(v for v in d["check"].values() if isinstance(v, bool)), d["check"]
+    if "--scaling" not in extra:
+        assert sum(d["check"]["spots_per_rank"]) == 64
+    if "warmup" in extra:
+        w = d["warmup_split"]
+        assert w["times_s"][0] > w["times_s"][1] and w["shares"][0] < w["shares"][1]   # rank 0 is slowed down
 
 
 def test_cpu_baseline_sample_sweep_library():
@@ -58,7 +70,15 @@ def test_cpu_baseline_sample_sweep_library():
     assert prob.cfg.n_lig == 0
     prob.lig = prob.ligands[0]
     lens = bench.list_lengths_host(prob, 12.0)
-    dt, pairs, poses, cores = bench.oracle_sample(prob, {"cutoff": 12.0}, {"preset": 3, "population": 64},
-                                                  lens, 0, 2, 1)
-    assert dt > 0 and cores >= 1 and poses > 0 and poses % 2 == 0
-    assert pairs == (int(lens[0]) + int(lens[1])) * len(prob.lig.q) * (poses // 2)
+    r = bench.oracle_sample(prob, {"cutoff": 12.0}, {"preset": 3, "population": 64}, lens, 0, 2, 1)
+    assert r["s"] > 0 and r["cores"] >= 1 and r["poses"] > 0 and r["poses"] % 2 == 0
+    assert r["pairs"] == (int(lens[0]) + int(lens[1])) * len(prob.lig.q) * (r["poses"] // 2)
+    assert 0 < r["within"] < r["pairs"] < r["visited"]
+
+
+def test_hetero_and_splits_helpers():
+    sys.path.insert(0, ROOT)
+    import bench
+    assert bench.hetero_factor("0:2,3:4", 0) == 2 and bench.hetero_factor("0:2,3:4", 3) == 4
+    assert bench.hetero_factor("", 1) == 1
+    assert bench.auto_splits(500) == 1 and bench.auto_splits(250) == 2 and bench.auto_splits(63) == 4

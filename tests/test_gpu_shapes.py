@@ -1,0 +1,155 @@
+"""Launch shapes never change a result; the instrumentation counts what it claims.
+
+The pair kernel cuts a scoring launch into warps by a launch shape (KP item pairs per lane: 64 KP items per chunk;
+one warp per chunk and canonical list split) chosen per launch for speed (vs_api.cu choose_shape).  An item's
+energy is the fixed fp64 tree (e_0 + e_1) + (e_2 + e_3) of its S split energies whatever the shape (vs_cells.cu
+header), so scores, vs_run results and the scores of vs_score_poses vs vs_run are bitwise identical across shapes.
+VS_SHAPE=kp (read at vs_create) forces a shape for these tests.
+"""
+import os
+
+import numpy as np
+import pytest
+
+from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
+
+pytestmark = pytest.mark.gpu
+SHAPES = {1: ["2", "1"], 2: ["2", "1"], 4: ["2", "1"]}
+
+
+@pytest.fixture(scope="module")
+def torch():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch
+
+
+def ctx_with_shape(prob, shape, S=1, **sp):
+    old = os.environ.get("VS_SHAPE")
+    if shape:
+        os.environ["VS_SHAPE"] = shape
+    try:
+        return vs.Context.from_problem(prob, vs.score_params(list_splits=S, **sp))
+    finally:
+        if old is None:
+            os.environ.pop("VS_SHAPE", None)
+        else:
+            os.environ["VS_SHAPE"] = old
+
+
+@pytest.mark.parametrize("S", [1, 2, 4])
+@pytest.mark.parametrize("cutoff", [12.0, 0.0])
+@pytest.mark.parametrize("name", ["small", "custom_hb"])
+def test_scores_bitwise_across_shapes(torch, oracle_mod, name, cutoff, S):
+    if name == "custom_hb":          # every H-bond slot layout: H-bond-heavy ligand (H = 2 at KP 2)
+        prob = synth.make_custom(2500, 23, 6, seed=17)
+        rng = np.random.default_rng(5)
+        prob.lig.type[:] = rng.choice([synth.T_N, synth.T_O, synth.T_HD, synth.T_HD, synth.T_C],
+                                      size=len(prob.lig.type)).astype(np.int32)
+    else:
+        prob = synth.make_problem(name)
+    spot, q, t = synth.make_poses(3000, prob.cfg.n_spots, 3.0, seed=13)
+    t[:1000] *= 0.3
+    ref = None
+    for sh in SHAPES[S]:
+        got = ctx_with_shape(prob, sh, S, cutoff=cutoff).score_poses(spot, q, t)
+        if ref is None:
+            ref = got
+            o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params(cutoff=cutoff))
+            idx = np.arange(0, len(spot), 150)
+            r = o.score(spot[idx], q[idx], t[idx])
+            assert np.all(np.abs(got[idx] - r) <= np.maximum(1e-4 * np.abs(r), 1e-3))
+        np.testing.assert_array_equal(got, ref, err_msg=f"shape {sh}")
+
+
+@pytest.mark.parametrize("S", [1, 4])
+def test_run_bitwise_across_shapes_and_entry_points(torch, S):
+    prob = synth.make_problem("small")
+    mp = vs.mh_preset(3, population=64, generations=3)
+    ref = None
+    for sh in [None] + SHAPES[S]:
+        g = ctx_with_shape(prob, sh, S)
+        p, s = g.run(mp, 17)
+        if ref is None:
+            ref = (p, s)
+            # the best score of a run is the score vs_score_poses gives its pose (a pose's score is a function of
+            # the pose alone)
+            again = g.score_poses(np.arange(prob.cfg.n_spots, dtype=np.int32), p[:, :4], p[:, 4:])
+            np.testing.assert_array_equal(again, s)
+        else:
+            np.testing.assert_array_equal(p, ref[0], err_msg=f"shape {sh}")
+            np.testing.assert_array_equal(s, ref[1], err_msg=f"shape {sh}")
+
+
+def test_list_splits_change_only_rounding(torch, oracle_mod):
+    """S = 1, 2, 4 canonical splits: a summation order; every variant within the tolerance of the oracle and within
+    fp32 rounding of each other."""
+    prob = synth.make_problem("small")
+    spot, q, t = synth.make_poses(2000, prob.cfg.n_spots, 3.0, seed=21)
+    got = {S: vs.Context.from_problem(prob, vs.score_params(list_splits=S)).score_poses(spot, q, t) for S in (1, 2, 4)}
+    o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params())
+    idx = np.arange(0, 2000, 40)
+    r = o.score(spot[idx], q[idx], t[idx])
+    for S, v in got.items():
+        assert np.all(np.abs(v[idx] - r) <= np.maximum(1e-4 * np.abs(r), 1e-3)), S
+        assert np.all(np.abs(v - got[1]) <= 1e-5 * np.maximum(np.abs(got[1]), 1.0)), S
+    assert not np.array_equal(got[4], got[1])           # a different (valid) rounding
+    with pytest.raises(vs.VSError):
+        vs.Context.from_problem(prob, vs.score_params(list_splits=3))
+
+
+def test_census_counts_pairs_within_cutoff(torch, oracle_mod):
+    """VS_TIMING_CENSUS: pairs_within equals the oracle's count of pairs with r^2 < rc^2 (the decision is taken in
+    fp32 on the GPU and fp64 in the oracle: pairs within rounding of rc may differ), scores bitwise unchanged."""
+    prob = synth.make_problem("small")
+    g = vs.Context.from_problem(prob, vs.score_params())
+    o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params())
+    spot, q, t = synth.make_poses(400, prob.cfg.n_spots, 3.0, seed=2)
+    plain = g.score_poses(spot, q, t)
+    g.reset_stats()
+    g.set_timing(vs.TIMING_CENSUS)
+    cen = g.score_poses(spot, q, t)
+    st = g.stats()
+    np.testing.assert_array_equal(cen, plain)
+    o.score(spot, q, t)
+    want = o.pairs_within()
+    assert abs(st["pairs_within"] - want) <= 2 + 1e-6 * want, (st["pairs_within"], want)
+    g.set_timing(0)
+    g.reset_stats()
+    g.score_poses(spot, q, t)
+    ev = g.stats()["pairs_evaluated"]                  # census launches count within-rc pairs instead
+    assert st["pairs_within"] < ev < st["pairs"]
+    # a census run gives the same result as a plain one
+    mp = vs.mh_preset(3, population=32, generations=2)
+    g.set_timing(0)
+    p0, s0 = g.run(mp, 3)
+    g.set_timing(vs.TIMING_CENSUS)
+    p1, s1 = g.run(mp, 3)
+    np.testing.assert_array_equal(s0, s1)
+
+
+def test_kernel_intervals_inside_graph_replays(torch):
+    """VS_TIMING_KERNEL records every pair-kernel launch interval, also in replayed CUDA graphs."""
+    prob = synth.make_problem("small")
+    g = vs.Context.from_problem(prob, vs.score_params())
+    mp = vs.mh_preset(3, population=64, generations=2)
+    g.set_timing(vs.TIMING_KERNEL)
+    st = torch.cuda.Stream()
+    bp = torch.empty((prob.cfg.n_spots, 7), device="cuda")
+    bs = torch.empty(prob.cfg.n_spots, device="cuda")
+    for _ in range(2):                     # direct, then captured
+        g.run_async(mp, 1, None, bp, bs, st)
+    st.synchronize()
+    g.reset_stats()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    for _ in range(3):                     # replays
+        g.run_async(mp, 1, None, bp, bs, st)
+    e1.record(st)
+    st.synchronize()
+    s = g.stats()
+    wall = e0.elapsed_time(e1)
+    assert s["pair_timed_launches"] == s["score_launches"] > 0
+    assert 0 < s["pair_busy_ms"] <= wall * 1.01 + 0.05
+    assert s["pair_launch_ms"] >= s["pair_busy_ms"] * 0.999

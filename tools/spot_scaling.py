@@ -23,19 +23,23 @@ def main():
     ap.add_argument("--generations", type=int, default=None)
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--ranks", default="1,2,4,8")
+    ap.add_argument("--spots", default=None, help="explicit spot counts instead of n_spots / ranks")
+    ap.add_argument("--splits", type=int, default=1, help="vs_score_params.list_splits")
     args = ap.parse_args()
     import numpy as np
     import torch
     from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
     prob = synth.make_problem(args.config)
     G = prob.cfg.generations if args.generations is None else args.generations
-    ctx = vs.Context.from_problem(prob, vs.score_params(), device=0)
+    ctx = vs.Context.from_problem(prob, vs.score_params(list_splits=args.splits), device=0)
     mp = vs.mh_preset(args.preset, population=prob.cfg.population, generations=G)
     st = torch.cuda.Stream()
     ns = prob.cfg.n_spots
     out = {}
-    for N in [int(x) for x in args.ranks.split(",")]:
-        n = (ns + N - 1) // N
+    counts = ([(ns + N - 1) // N for N in map(int, args.ranks.split(","))] if args.spots is None
+              else [int(x) for x in args.spots.split(",")])
+    for n in counts:
+        N = ns / n
         ids = np.arange(n, dtype=np.int32)
         bp = torch.empty((n, 7), device="cuda")
         bs = torch.empty(n, device="cuda")
@@ -48,11 +52,12 @@ def main():
             ctx.run_async(mp, 42, ids, bp, bs, st)
         e1.record(st)
         torch.cuda.synchronize()
-        out[N] = {"spots": n, "ms": e0.elapsed_time(e1) / args.reps}
-    t1 = out[min(out)]["ms"]
-    for N, v in out.items():
-        v["eff"] = t1 / (N * v["ms"])
-    print(json.dumps({"config": args.config, "generations": G, "T": out}))
+        out[n] = {"N": N, "ms": e0.elapsed_time(e1) / args.reps}
+    if ns in out:
+        t1 = out[ns]["ms"]
+        for n, v in out.items():
+            v["eff"] = t1 / (v["N"] * v["ms"])
+    print(json.dumps({"config": args.config, "generations": G, "list_splits": args.splits, "T": out}))
     ctx.close()
 
 
