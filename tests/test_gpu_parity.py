@@ -365,12 +365,14 @@ def test_run_errors(gpu, oracle_mod):
         g.run(vs.mh_preset(1, population=4096), 1)
 
 
-@pytest.mark.parametrize("preset,P,G,K", [(3, 32, 4, 1), (2, 16, 2, 1), (4, 64, 0, 1), (3, 32, 2, 2), (4, 64, 0, 3)])
-def test_lockstep_trace(gpu, oracle_mod, preset, P, G, K):
+@pytest.mark.parametrize("preset,P,G,K,cutoff", [(3, 32, 4, 1, 12.0), (2, 16, 2, 1, 12.0), (4, 64, 0, 1, 12.0),
+                                                (3, 32, 2, 2, 12.0), (4, 64, 0, 3, 12.0),
+                                                (3, 32, 3, 1, 0.0), (4, 64, 0, 2, 0.0)])
+def test_lockstep_trace(gpu, oracle_mod, preset, P, G, K, cutoff):
     """Every stage of Algorithm 1 on the GPU re-derived by the oracle from the GPU's own state:
     pose generation byte-exact, decisions exact on GPU scores, scores within tolerance.
-    K > 1: parallel-neighbourhood Improve (best of K proposals per step, N4)."""
-    prob, (g, o) = _run_pair(oracle_mod)
+    K > 1: parallel-neighbourhood Improve (best of K proposals per step, N4); cutoff 0: all-pairs (paper) mode."""
+    prob, (g, o) = _run_pair(oracle_mod, cutoff=cutoff)
     seed = 77
     mp_g = vs.mh_preset(preset, population=P, generations=G, ls_neighbours=K)
     mp_o = oracle_mod.mh_preset(preset, population=P, generations=G, ls_neighbours=K)
