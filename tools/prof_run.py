@@ -1,9 +1,10 @@
 #!/usr/bin/env python
-"""Profiling driver: one vs_run of a config (direct launches) for ncu, e.g.
+"""Profiling driver: one vs_run of a config for ncu, e.g.
 
   VS_GRAPHS=0 ncu --set full -k regex:cell_pair_kernel -c 2 -o gpurun_out/pair python tools/prof_run.py --generations 1
-
-Runs one warm-up call first when --warm is given (so that lazy module loading is outside the capture).
+  ncu --graph-profiling graph --metrics ... python tools/prof_run.py --generations 10 --graph
+      (--graph: a direct run, a captured run, then one replay of the CUDA graph -- the in-run workload of the bench,
+       all spot-group streams concurrent -- which ncu profiles as one workload)
 """
 import argparse
 import os
@@ -11,6 +12,7 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 
 
 def main():
@@ -19,6 +21,7 @@ def main():
     ap.add_argument("--preset", type=int, default=3)
     ap.add_argument("--generations", type=int, default=1)
     ap.add_argument("--score-poses", type=int, default=0, help="also score N random poses via vs_score_poses")
+    ap.add_argument("--graph", action="store_true", help="direct run, captured run, then one graph replay")
     args = ap.parse_args()
     import torch
     from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
@@ -26,6 +29,10 @@ def main():
     g = vs.Context.from_problem(prob, vs.score_params(), device=0)
     mp = vs.mh_preset(args.preset, population=prob.cfg.population, generations=args.generations)
     g.run(mp, 42)
+    if args.graph:
+        g.run(mp, 42)          # captured
+        torch.cuda.synchronize()
+        g.run(mp, 42)          # replayed
     if args.score_poses:
         spot, q, t = synth.make_poses(args.score_poses, prob.cfg.n_spots, 3.0, seed=1)
         g.score_poses(spot, q, t)
