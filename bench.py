@@ -187,8 +187,9 @@ def hetero_factor(spec: str, rank: int) -> int:
 
 def auto_splits(n_spots_per_rank: int) -> int:
     """Canonical list splits for a run of this many spots per GPU: latency-bound runs (few spots) get more
-    warps per chunk (profiles/r02_notes.md: medium at 63 spots / GPU 115 -> 87 ms with 4 splits)."""
-    return 4 if n_spots_per_rank <= 128 else (2 if n_spots_per_rank <= 256 else 1)
+    warps per chunk (profiles/r02_notes.md, medium: 63 spots 105.6 -> 85.2 ms with 4 splits, 125 spots 159.7 ->
+    140.3 ms with 2, 250 spots best with 1)."""
+    return 4 if n_spots_per_rank <= 96 else (2 if n_spots_per_rank <= 200 else 1)
 
 
 # ---------------------------------------------------------------- oracle arm / cpu baseline

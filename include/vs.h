@@ -79,7 +79,7 @@ typedef struct {
   const float* type_eps;      /* [n_types] kcal/mol (>= 0) */
   const int* type_hb_role;    /* [n_types] 0 none, 1 donor, 2 acceptor */
   int list_splits;            /* canonical receptor-list splits S: 1, 2 or 4; 0 (default) = by the spot count
-                                 (<= 128 spots: 4, <= 256: 2, else 1).  The GPU sums each
+                                 (<= 96 spots: 4, <= 200: 2, else 1).  The GPU sums each
                                  split's pairs in fp32 and combines the split energies of an atom by the fixed fp64
                                  tree (e0 + e1) + (e2 + e3): a summation order, so scores differ from S = 1 at fp32
                                  rounding (all within the tolerance).  For a given S a pose's score is the same from

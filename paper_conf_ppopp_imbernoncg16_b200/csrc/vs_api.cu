@@ -196,6 +196,9 @@ static_assert(vsk::CELL_G % vsk::CELL_NSPLIT == 0, "the pair kernel assigns cell
 #ifndef VS_FILL_WARPS
 #define VS_FILL_WARPS 2048    // pair-kernel warps below which a scoring round uses KP = 1 chunks (launch shape)
 #endif
+#ifndef VS_DIRECT_GROUP_SPOTS
+#define VS_DIRECT_GROUP_SPOTS 16  // un-graphed runs: spots per stream group at least (small e2e 34 -> 24 ms / step)
+#endif
 #ifndef VS_GRAPH_CACHE
 #define VS_GRAPH_CACHE 4      // CUDA graphs kept per context
 #endif
@@ -235,6 +238,7 @@ struct vs_ctx {
   long long fill_warps = VS_FILL_WARPS;  // launch shape target (speed only)
   int nsplit = 1;                        // canonical receptor-list splits (vs_score_params.list_splits)
   int force_kp = 0;                      // VS_SHAPE=kp (experiments)
+  int direct_group_spots = VS_DIRECT_GROUP_SPOTS;  // spots per stream group at least, un-graphed runs
   float4* d_ligx = nullptr;             // [n_lig] centred local coordinates, w = class
   float4* d_ligp = nullptr;             // [n_lig] es, c12, c6, donor
   int* d_lig_rank = nullptr;            // [n_lig] rank within the class
@@ -555,6 +559,9 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
   // un-graphed run (host-bound: 16 streams doubled it on the small config), hence >= 8 spots per group.
   int G = std::max(1, std::min(NSUB, ns / VS_GROUP_SPOTS));
   if (ns >= VS_BIG_RUN_SPOTS) G = std::min(G, VS_BIG_RUN_GROUPS);
+  // a run enqueued launch by launch (not captured into a graph: a context's first call) is bound by the host's
+  // launch rate when it has few spots per group: fewer groups, fewer launches (results do not depend on grouping)
+  if (!c->capturing) G = std::max(1, std::min(G, ns / c->direct_group_spots));
   if (tr) G = 1;
   Group grp[NSUB];
   CK(cudaEventRecord(c->ev_fork, st), "event record");
@@ -879,7 +886,7 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
       !(sp.r2_min > 0.0f && std::isfinite(sp.r2_min)) || std::isnan(sp.cutoff))
     return set_err(VS_ERR_INVALID_ARGUMENT, "invalid score params");
   // list_splits 0 = by the context's spot count: few spots -> latency-bound runs -> more splits (R32)
-  if (sp.list_splits == 0) sp.list_splits = n_spots <= 128 ? 4 : (n_spots <= 256 ? 2 : 1);
+  if (sp.list_splits == 0) sp.list_splits = n_spots <= 96 ? 4 : (n_spots <= 200 ? 2 : 1);
   if (sp.list_splits != 1 && sp.list_splits != 2 && sp.list_splits != 4)
     return set_err(VS_ERR_INVALID_ARGUMENT, "list_splits must be 0, 1, 2 or 4");
   if (sp.n_types < 0 || sp.n_types > 64 || (sp.n_types > 0 && (!sp.type_sigma || !sp.type_eps || !sp.type_hb_role)))
@@ -926,6 +933,7 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   c->n_spots = n_spots;
   // launch-shape knobs for experiments (speed only; results never depend on them)
   if (const char* v = std::getenv("VS_FILL_WARPS")) c->fill_warps = std::max(1ll, std::atoll(v));
+  if (const char* v = std::getenv("VS_DIRECT_GROUP_SPOTS")) c->direct_group_spots = std::max(1, std::atoi(v));
   if (const char* v = std::getenv("VS_SHAPE")) {  // "kp"
     const int kp = std::atoi(v);
     if (kp == 1 || kp == 2) c->force_kp = kp;

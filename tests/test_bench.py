@@ -81,4 +81,4 @@ def test_hetero_and_splits_helpers():
     import bench
     assert bench.hetero_factor("0:2,3:4", 0) == 2 and bench.hetero_factor("0:2,3:4", 3) == 4
     assert bench.hetero_factor("", 1) == 1
-    assert bench.auto_splits(500) == 1 and bench.auto_splits(250) == 2 and bench.auto_splits(63) == 4
+    assert bench.auto_splits(500) == 1 and bench.auto_splits(250) == 1 and bench.auto_splits(125) == 2 and bench.auto_splits(63) == 4
