@@ -808,17 +808,11 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
 // vs_score_poses_device and a vs_run_async of the same ctx), and graph capture always happens on a capturable
 // (non-legacy) stream whatever the caller passes (NULL = the legacy default stream included).
 vs_status join_in(vs_ctx* c, cudaStream_t caller) {
-#ifdef VS_NO_JOIN
-  return VS_OK;
-#endif
   CK(cudaEventRecord(c->ev_in, caller), "event record (caller stream)");
   CK(cudaStreamWaitEvent(c->stream, c->ev_in, 0), "stream wait");
   return VS_OK;
 }
 vs_status join_out(vs_ctx* c, cudaStream_t caller) {
-#ifdef VS_NO_JOIN
-  return VS_OK;
-#endif
   CK(cudaEventRecord(c->ev_out, c->stream), "event record");
   CK(cudaStreamWaitEvent(caller, c->ev_out, 0), "stream wait (caller stream)");
   return VS_OK;
@@ -1228,11 +1222,7 @@ vs_status vs_run_async(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t
   if (!d_best_pose || !d_best_score) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL output");
   DeviceGuard guard(c->dev);
   vs_status r = join_in(c, (cudaStream_t)stream);
-#ifdef VS_NO_JOIN
-  if (r == VS_OK) r = run_impl(c, mp, seed, n_sel, spot_ids, d_best_pose, d_best_score, (cudaStream_t)stream, nullptr);
-#else
   if (r == VS_OK) r = run_impl(c, mp, seed, n_sel, spot_ids, d_best_pose, d_best_score, c->stream, nullptr);
-#endif
   if (r == VS_OK) r = join_out(c, (cudaStream_t)stream);
   return r;
 }
