@@ -337,6 +337,7 @@ vs_status collect_timing(vs_ctx* c) {
 // measured slower than one warp per split even for latency-bound launches: profiles/r02_notes.md.)
 struct Shape {
   int kp, H, cn, chb, w, S;
+  int nn, nh, merged;  // item classes of the launch (merged: every atom in the H-bond class, one curve order)
   int nsg() const { return S; }
 };
 Shape shape_of(const vs_ctx* c, int kp, int w) {
@@ -347,12 +348,22 @@ Shape shape_of(const vs_ctx* c, int kp, int w) {
   s.cn = 64 * kp;
   s.chb = 64 * s.H;
   s.w = w;
+  s.nn = c->nn;
+  s.nh = c->nh;
+  s.merged = 0;
+  // a KP = 1 chunk has one slot pair, an H-bond pair whenever the ligand has H-bond atoms: its items then go in one
+  // class and one curve order (spatially tighter chunks at no extra cost per pair; layout only, never a result)
+  if (kp == 1 && s.H == 1 && c->nn > 0) {
+    s.nn = 0;
+    s.nh = c->n_lig;
+    s.merged = 1;
+  }
   return s;
 }
 Shape choose_shape(const vs_ctx* c, long long n_seg, int seg_n) {
   if (c->force_kp) return shape_of(c, c->force_kp, 1);
   const Shape s2 = shape_of(c, 2, 1);
-  if (n_seg * cell_chunks(seg_n, c->nn, c->nh, s2.cn, s2.chb) * s2.nsg() >= c->fill_warps) return s2;
+  if (n_seg * cell_chunks(seg_n, s2.nn, s2.nh, s2.cn, s2.chb) * s2.nsg() >= c->fill_warps) return s2;
   return shape_of(c, 1, 1);
 }
 void apply_shape(CellArgs& a, const Shape& s) {
@@ -362,6 +373,9 @@ void apply_shape(CellArgs& a, const Shape& s) {
   a.chb = s.chb;
   a.w = s.w;
   a.nsplit = s.S;
+  a.nn = s.nn;
+  a.nh = s.nh;
+  a.merged = s.merged;
 }
 
 CellArgs cell_base(vs_ctx* c) {
@@ -378,8 +392,6 @@ CellArgs cell_base(vs_ctx* c) {
   a.ligp = c->d_ligp;
   a.lig_rank = c->d_lig_rank;
   a.n_lig = c->n_lig;
-  a.nn = c->nn;
-  a.nh = c->nh;
   apply_shape(a, shape_of(c, 2, 4));
   a.shift = c->d_shift;
   a.W = c->W;
@@ -589,7 +601,7 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
       cp.seg_stride = P;
       cp.P = P;
       cp.mode = MODE_PLAIN;
-      cp.nch_u = cell_chunks(P, c->nn, c->nh, shp.cn, shp.chb);
+      cp.nch_u = cell_chunks(P, shp.nn, shp.nh, shp.cn, shp.chb);
       cp.pbuf = b.pbuf + (size_t)k0 * maxpose;
       cp.items = b.items + (size_t)k0 * maxpose * c->n_lig;
       cp.E = b.E + (size_t)k0 * c->n_lig * b.emax;
@@ -599,7 +611,7 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
       apply_shape(cl, shl);
       cl.mode = MODE_LS;
       cl.seg_size = mk;
-      cl.nch_u = cell_chunks(mk, c->nn, c->nh, shl.cn, shl.chb);
+      cl.nch_u = cell_chunks(mk, shl.nn, shl.nh, shl.cn, shl.chb);
       cl.E_stride = (long long)q.ns * mk * c->n_lig;
       cl.J = q.J;
       cl.m = m;
@@ -770,7 +782,7 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
     int* orig = (int*)c->buf[B_ORIG].p;
     CK(cudaMemsetAsync(counts, 0, sizeof(int) * ns, st), "memset");
     CK(launch_validate(nb, sp, q, t, ns, c->T, c->all_pairs ? 0 : 1, valid, counts, out, st), "validate launch");
-    CK(launch_cell_scan(counts, ns, c->nn, c->nh, sh.cn, sh.chb, pp, cp, cur, st), "scan launch");
+    CK(launch_cell_scan(counts, ns, sh.nn, sh.nh, sh.cn, sh.chb, pp, cp, cur, st), "scan launch");
     CK(launch_scatter(nb, sp, q, t, valid, cur, sorted, orig, st), "scatter launch");
     c->launches += 3;
     CellArgs a = cell_base(c);
@@ -790,7 +802,7 @@ vs_status score_device_cells(vs_ctx* c, int64_t n, const int32_t* d_spot, const 
     a.E_stride = nb * c->n_lig;
     // pair-kernel grid: an upper bound of sum_k cell_chunks(n_k) (<= n_k n_lig / cn + n_k nh / chb + 3)
     int64_t blocks = 3 * (int64_t)ns + (nb * c->n_lig) / sh.cn + 1;
-    if (sh.chb > 0) blocks += (nb * c->nh) / sh.chb;
+    if (sh.chb > 0) blocks += (nb * sh.nh) / sh.chb;
     blocks *= sh.nsg();
     if (blocks > 0x7fffffff) return set_err(VS_ERR_INVALID_ARGUMENT, "too many poses in one call");
     vs_status r = cell_launch(c, a, nb, (int)blocks, st);
@@ -982,7 +994,13 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     int cnt[2] = {0, 0};
     bool any_role = false;  // a ligand without H-bond atoms keeps H = 0 (no H-bond slots) even with VS_CELL_MERGE
     for (int i = 0; i < n_lig; ++i) any_role = any_role || don[lig_type[i]] != 0.0f || acc[lig_type[i]] != 0.0f;
-    const bool merge = VS_CELL_MERGE && any_role;
+    // one item class for every launch ("merge": every atom in the H-bond slots, one curve order, spatially tighter
+    // slot pairs at 23 instead of 19 issue slots for class-0 pairs): measured large -2.5 %, medium +2.3 %, sweep
+    // +2.5 % (profiles/r02_notes.md), so off by default; KP = 1 launches merge anyway (shape_of).  Layout only: the
+    // item order never enters a result.  VS_CELL_MERGE=0/1 (environment) forces it.
+    int merge_mode = VS_CELL_MERGE;
+    if (const char* v = std::getenv("VS_CELL_MERGE")) merge_mode = std::atoi(v);
+    const bool merge = merge_mode && any_role;
     for (int i = 0; i < n_lig; ++i) {
       const int t = lig_type[i];
       const int role = (don[t] != 0.0f || acc[t] != 0.0f) ? 1 : 0;

@@ -91,7 +91,8 @@ struct CellArgs {
   const float4* ligx;        // local x, y, z (centred), w = class (0: class 0; 1: class 1, donor / acceptor; 2: class 1, no role)
   const float4* ligp;        // es_i, c12_i, c6_i, donor_i
   const int* lig_rank;       // rank of the atom within its class
-  int n_lig, nn, nh;         // atoms, of which nn without / nh with an H-bond role
+  int n_lig, nn, nh;         // atoms; in class 0 / class 1 (H-bond role) for this launch (merged: 0 / n_lig)
+  int merged;                // every atom in class 1, rank = atom index (a KP = 1 launch of a ligand with roles)
   // launch shape (speed only, never results): kp packed item pairs per lane (1 or 2), H of them H-bond pairs (the
   // first kp - H pairs hold class 0 only), chunk capacities cn = 64 kp items, chb = 64 H class-1 items (w: 1)
   int kp, H, cn, chb, w;

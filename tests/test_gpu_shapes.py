@@ -82,6 +82,31 @@ def test_run_bitwise_across_shapes_and_entry_points(torch, S):
             np.testing.assert_array_equal(s, ref[1], err_msg=f"shape {sh}")
 
 
+@pytest.mark.parametrize("name", ["small", "medium"])
+def test_item_class_layout_bitwise(torch, name):
+    """The merged item layout (every ligand atom in the H-bond slots, one curve order: the default for ligands with at
+    most a third of H-bond atoms) and the class-separated layout give bitwise identical scores and runs."""
+    prob = synth.make_problem(name)
+    spot, q, t = synth.make_poses(2000, prob.cfg.n_spots, 3.0, seed=4)
+    mp = vs.mh_preset(3, population=32, generations=2)
+    ids = np.arange(min(prob.cfg.n_spots, 16), dtype=np.int32)
+    res = []
+    for m in ("0", "1"):
+        old = os.environ.get("VS_CELL_MERGE")
+        os.environ["VS_CELL_MERGE"] = m
+        try:
+            g = vs.Context.from_problem(prob, vs.score_params())
+        finally:
+            if old is None:
+                os.environ.pop("VS_CELL_MERGE", None)
+            else:
+                os.environ["VS_CELL_MERGE"] = old
+        res.append((g.score_poses(spot, q, t), g.run(mp, 9, ids)))
+    np.testing.assert_array_equal(res[0][0], res[1][0])
+    np.testing.assert_array_equal(res[0][1][0], res[1][1][0])
+    np.testing.assert_array_equal(res[0][1][1], res[1][1][1])
+
+
 def test_list_splits_change_only_rounding(torch, oracle_mod):
     """S = 1, 2, 4 canonical splits: a summation order; every variant within the tolerance of the oracle and within
     fp32 rounding of each other."""
