@@ -178,3 +178,64 @@ def test_kernel_intervals_inside_graph_replays(torch):
     assert s["pair_timed_launches"] == s["score_launches"] > 0
     assert 0 < s["pair_busy_ms"] <= wall * 1.01 + 0.05
     assert s["pair_launch_ms"] >= s["pair_busy_ms"] * 0.999
+
+
+def test_graph_cache_keeps_several_shapes(torch):
+    """Runs of a few chunk sizes (a multi-GPU queue's chunks) each replay their own CUDA graph (LRU of 4): results
+    equal direct launches bit for bit whatever the interleaving."""
+    prob = synth.make_problem("small")
+    g = vs.Context.from_problem(prob, vs.score_params())
+    mp = vs.mh_preset(3, population=32, generations=2)
+    chunks = [np.arange(0, 10, dtype=np.int32), np.arange(10, 30, dtype=np.int32), np.arange(30, 64, dtype=np.int32),
+              np.arange(5, 12, dtype=np.int32), np.arange(40, 45, dtype=np.int32)]
+    ref = [g.run(mp, 3, ids) for ids in chunks]                  # direct launches (first sight of each shape)
+    st = torch.cuda.Stream()
+    for rep in range(3):                                          # second sight captures, then replays; 5 shapes > 4
+        for ids, (rp, rs) in zip(chunks, ref):
+            bp = torch.empty((len(ids), 7), device="cuda")
+            bs = torch.empty(len(ids), device="cuda")
+            g.run_async(mp, 3, ids, bp, bs, st)
+            st.synchronize()
+            np.testing.assert_array_equal(bs.cpu().numpy(), rs)
+            np.testing.assert_array_equal(bp.cpu().numpy(), rp)
+
+
+def test_long_lists_and_splits(torch, oracle_mod):
+    """Lists streamed whole (> 16384 atoms: cut by position into the S canonical splits) give the same scores for
+    every S within fp32 rounding and the oracle's within tolerance; the census counts them."""
+    prob = synth.make_custom(25000, 30, 3, seed=23)
+    spot, q, t = synth.make_poses(120, 3, 3.0, seed=4)
+    o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params(cutoff=70.0))
+    ref = o.score(spot, q, t)
+    for S in (1, 2, 4):
+        g = vs.Context.from_problem(prob, vs.score_params(cutoff=70.0, list_splits=S))
+        assert g.list_lengths().max() > 16384
+        got = g.score_poses(spot, q, t)
+        assert np.all(np.abs(got - ref) <= np.maximum(1e-4 * np.abs(ref), 1e-3)), S
+        g.set_timing(vs.TIMING_CENSUS)
+        g.reset_stats()
+        np.testing.assert_array_equal(g.score_poses(spot, q, t), got)
+        assert g.stats()["pairs_within"] > 0
+
+
+def test_census_all_pairs_counts_every_pair(torch):
+    prob = synth.make_problem("tiny")
+    g = vs.Context.from_problem(prob, vs.score_params(cutoff=0.0))
+    g.set_timing(vs.TIMING_CENSUS)
+    g.reset_stats()
+    spot, q, t = synth.make_poses(50, prob.cfg.n_spots, 3.0, seed=1)
+    g.score_poses(spot, q, t)
+    st = g.stats()
+    assert st["pairs_within"] == st["pairs"] == 50 * prob.cfg.n_rec * prob.cfg.n_lig
+
+
+def test_no_hbond_ligand_kp1(torch, oracle_mod):
+    """A ligand without H-bond atoms (H = 0: no H-bond slot pairs at KP 1 or 2) through both shapes and a run."""
+    prob = synth.make_custom(2500, 23, 6, seed=17)
+    prob.lig.type[:] = synth.T_C
+    spot, q, t = synth.make_poses(500, 6, 3.0, seed=2)
+    res = [ctx_with_shape(prob, sh, 1).score_poses(spot, q, t) for sh in ("2", "1")]
+    np.testing.assert_array_equal(res[0], res[1])
+    o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params())
+    r = o.score(spot[:60], q[:60], t[:60])
+    assert np.all(np.abs(res[0][:60] - r) <= np.maximum(1e-4 * np.abs(r), 1e-3))
