@@ -488,15 +488,15 @@ def main():
 
     # the pair kernel's launch intervals are recorded in the warm-up steps too: the instrumented launches are what
     # the warm-up captures into the CUDA graphs the timed steps replay
-    work_ctx = list(scr.ctx.values()) if sweep else runner.ctx
-    for c in work_ctx:
-        c.set_timing(vs.TIMING_KERNEL)
+    if sweep:
+        scr.set_timing(vs.TIMING_KERNEL)        # also for the contexts the sweep creates lazily
+    else:
+        runner.set_timing(vs.TIMING_KERNEL)
     for i in range(args.warmup):
         step(-1 - i)
     torch.cuda.synchronize(dev)
     work_ctx = list(scr.ctx.values()) if sweep else runner.ctx   # the sweep creates its contexts lazily
     for c in work_ctx:
-        c.set_timing(vs.TIMING_KERNEL)
         c.reset_stats()
     clocks = ClockSampler(local, enabled=(rank == 0 and not args.no_clocks))
     if world > 1:
@@ -513,11 +513,15 @@ def main():
         dist.barrier()
     clk = clocks.stop()
     ms_rank = e0.elapsed_time(e1)
+    work_ctx = list(scr.ctx.values()) if sweep else runner.ctx
     st = {}
     for c in work_ctx:
         for k, v in c.stats().items():
             st[k] = st.get(k, 0) + v
-        c.set_timing(0)
+    if sweep:
+        scr.set_timing(0)
+    else:
+        runner.set_timing(0)
     # whole-job totals and max-over-ranks time
     tot = torch.tensor([st["pairs"], st["poses_scored"], st["kernel_launches"], st["pairs_evaluated"]],
                        dtype=torch.float64, device=cdev)

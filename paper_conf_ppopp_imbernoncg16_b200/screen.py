@@ -57,13 +57,21 @@ class Screen:
         self.sp, self.mp, self.seed, self.device = sp, mp, seed, device
         self.ctx: dict[int, vs.Context] = {}
         self.done: list[tuple[int, int, int]] = []
+        self.timing = 0   # vs_set_timing flags given to every context, also those created later (lazily)
 
     def context(self, li: int) -> vs.Context:
         if li not in self.ctx:
             L = self.ligands[li]
             self.ctx[li] = vs.Context(self.rec.xyz, self.rec.q, self.rec.type, L.xyz, L.q, L.type, self.spots,
                                       self.sp, self.device)
+            if self.timing:
+                self.ctx[li].set_timing(self.timing)
         return self.ctx[li]
+
+    def set_timing(self, flags: int) -> None:
+        self.timing = flags
+        for c in self.ctx.values():
+            c.set_timing(flags)
 
     def prepare(self, ligs: Sequence[int]) -> None:
         for li in ligs:

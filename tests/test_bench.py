@@ -60,6 +60,15 @@ def test_bench_two_ranks_gloo_on_one_gpu(extra):
         assert w["times_s"][0] > w["times_s"][1] and w["shares"][0] < w["shares"][1]   # rank 0 is slowed down
 
 
+@pytest.mark.gpu
+def test_bench_sweep_two_ranks_gloo():
+    """The screening sweep (N1) through the multi-rank path: (ligand, spot chunk) units dealt by the queue, the
+    fixed-size [ligands x spots] record table gathered and checked per ligand against a single-process run."""
+    d = _run([sys.executable, "bench.py", "--gpus", "2", "--config", "sweep", "--steps", "1", "--warmup", "1",
+              "--generations", "2", "--no-micro", "--no-cpu-baseline", "--no-e2e"], env={"VS_BENCH_BACKEND": "gloo"})
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["check"]["assembled_equals_single_process"] is True
+
+
 def test_cpu_baseline_sample_sweep_library():
     """The cpu_baseline leg samples ligand 0 of a screening library (cfg.n_lig is 0 there): the pair count is
     n_lig(ligand 0) x list length x poses per spot, and the pose count is population x (1 + generations x steps)."""
