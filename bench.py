@@ -612,7 +612,12 @@ def main():
             "within_over_evaluated": frac_within,
             "pair_kernel_busy_ms_per_step": st["pair_busy_ms"] / args.steps,
             "pair_kernel_share_of_step": st["pair_busy_ms"] / max(1e-9, ms_rank),
-            "pair_kernel_launch_ms_sum": st["pair_launch_ms"], "pair_kernel_launches": st["pair_timed_launches"]}
+            "pair_kernel_launch_ms_sum": st["pair_launch_ms"], "pair_kernel_launches": st["pair_timed_launches"],
+            "pair_kernel_warps_per_sm_in_run": st["pair_warp_ms"] / max(1e-9, st["pair_busy_ms"]) / N_SM,
+            "pair_kernel_warps_per_sm_max": 20,
+            "in_run_basis": "sum over every pair-kernel warp of its globaltimer duration / busy time / 148 SMs: the "
+                            "average number of resident pair-kernel warps per SM during the timed steps (one-warp "
+                            "CTAs, 96 registers: at most 20)"}
     if clk:
         roof["frac_at_run_clock"] = roof["frac"] * f_max / clk["sm_mhz"]
 

@@ -196,6 +196,8 @@ typedef struct {
   double pair_launch_ms;     /* VS_TIMING_KERNEL: sum of the pair kernel's launch intervals (first warp start to
                                 last warp end, device globaltimer; concurrent launches overlap) */
   uint64_t pair_timed_launches;
+  double pair_warp_ms;       /* VS_TIMING_KERNEL: sum over every pair-kernel warp of its duration (warp-ms): divided by
+                                the busy time and the SM count, the average number of resident pair-kernel warps */
 } vs_stats;
 
 /* Instrumentation flags of vs_set_timing (OR-ed):

@@ -253,7 +253,7 @@ struct vs_ctx {
   // instrumentation
   uint64_t launches = 0, score_launches = 0;
   bool timing = false, ktime = false, census = false;
-  unsigned long long* d_kt = nullptr;       // [VS_KT_CAP][2] pair-kernel launch intervals (~start, end) in ns
+  unsigned long long* d_kt = nullptr;       // [VS_KT_CAP][KT_WORDS] pair-kernel launch intervals (~start, end, warp ns)
   unsigned long long* d_kt_base = nullptr;  // first slot of the next run's region
   int kt_local = 0;                         // slots used by the run being enqueued
   std::vector<cudaEvent_t> ev;  // pairs (start, end)
@@ -1316,9 +1316,9 @@ vs_status vs_set_timing(vs_ctx* c, int flags) {
   DeviceGuard guard(c->dev);
   if ((flags & VS_TIMING_KERNEL) && !c->d_kt) {
     CK(cudaStreamSynchronize(c->stream), "sync");
-    CK(pool::alloc(&c->d_kt, sizeof(unsigned long long) * 2 * (size_t)VS_KT_CAP), "alloc");
+    CK(pool::alloc(&c->d_kt, sizeof(unsigned long long) * KT_WORDS * (size_t)VS_KT_CAP), "alloc");
     CK(pool::alloc(&c->d_kt_base, sizeof(unsigned long long)), "alloc");
-    CK(cudaMemset(c->d_kt, 0, sizeof(unsigned long long) * 2 * (size_t)VS_KT_CAP), "memset");
+    CK(cudaMemset(c->d_kt, 0, sizeof(unsigned long long) * KT_WORDS * (size_t)VS_KT_CAP), "memset");
     CK(cudaMemset(c->d_kt_base, 0, sizeof(unsigned long long)), "memset");
   }
   c->timing = (flags & VS_TIMING_EVENTS) != 0;
@@ -1337,17 +1337,23 @@ vs_status vs_get_stats(vs_ctx* c, vs_stats* o) {
   unsigned long long h[4];
   CK(cudaMemcpy(h, c->d_counters, sizeof(h), cudaMemcpyDeviceToHost), "D2H counters");
   o->pairs_within = c->all_pairs ? h[2] : h[3];  // all-pairs mode: every pair is within
-  o->pair_busy_ms = o->pair_launch_ms = 0.0;
+  o->pair_busy_ms = o->pair_launch_ms = o->pair_warp_ms = 0.0;
   o->pair_timed_launches = 0;
   if (c->d_kt) {  // pair-kernel launch intervals: their sum and the length of their union
     unsigned long long nslot = 0;
     CK(cudaMemcpy(&nslot, c->d_kt_base, sizeof(nslot), cudaMemcpyDeviceToHost), "D2H kt");
     nslot = std::min<unsigned long long>(nslot, VS_KT_CAP);
-    std::vector<unsigned long long> kt(2 * nslot);
-    if (nslot) CK(cudaMemcpy(kt.data(), c->d_kt, sizeof(unsigned long long) * 2 * nslot, cudaMemcpyDeviceToHost), "D2H kt");
+    std::vector<unsigned long long> kt(KT_WORDS * nslot);
+    if (nslot)
+      CK(cudaMemcpy(kt.data(), c->d_kt, sizeof(unsigned long long) * KT_WORDS * nslot, cudaMemcpyDeviceToHost), "D2H kt");
     std::vector<std::pair<unsigned long long, unsigned long long>> iv;
+    double warp_ns = 0.0;
     for (unsigned long long i = 0; i < nslot; ++i)
-      if (kt[2 * i] && kt[2 * i + 1]) iv.emplace_back(~kt[2 * i], kt[2 * i + 1]);
+      if (kt[KT_WORDS * i] && kt[KT_WORDS * i + 1]) {
+        iv.emplace_back(~kt[KT_WORDS * i], kt[KT_WORDS * i + 1]);
+        warp_ns += (double)kt[KT_WORDS * i + 2];
+      }
+    o->pair_warp_ms = warp_ns * 1e-6;
     std::sort(iv.begin(), iv.end());
     double sum = 0.0, busy = 0.0;
     unsigned long long cs = 0, ce = 0;
@@ -1386,7 +1392,7 @@ vs_status vs_reset_stats(vs_ctx* c) {
   CK(cudaDeviceSynchronize(), "sync");
   CK(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 4), "memset");
   if (c->d_kt) {
-    CK(cudaMemset(c->d_kt, 0, sizeof(unsigned long long) * 2 * (size_t)VS_KT_CAP), "memset");
+    CK(cudaMemset(c->d_kt, 0, sizeof(unsigned long long) * KT_WORDS * (size_t)VS_KT_CAP), "memset");
     CK(cudaMemset(c->d_kt_base, 0, sizeof(unsigned long long)), "memset");
   }
   c->ev_used = 0;

@@ -134,6 +134,7 @@ struct CellArgs {
   const unsigned long long* kt_base;
   int kt_slot, kt_cap;
 };
+constexpr int KT_WORDS = 3;  // per launch slot: ~start, end, sum of warp durations (ns)
 
 // Chunks of a segment of seg_n poses: class-1 items (H-bond role) fill at most cap1 = 64 H slots (the last H
 // slot pairs of each lane), class-0 items the other slots and any H-bond slot left over; a chunk takes the

@@ -59,7 +59,7 @@ class Stats(C.Structure):
     _fields_ = [("kernel_launches", C.c_uint64), ("score_launches", C.c_uint64), ("poses_scored", C.c_uint64),
                 ("pairs", C.c_uint64), ("score_ms", C.c_double), ("timed_launches", C.c_uint64),
                 ("pairs_evaluated", C.c_uint64), ("pairs_within", C.c_uint64), ("pair_busy_ms", C.c_double),
-                ("pair_launch_ms", C.c_double), ("pair_timed_launches", C.c_uint64)]
+                ("pair_launch_ms", C.c_double), ("pair_timed_launches", C.c_uint64), ("pair_warp_ms", C.c_double)]
 
     def asdict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

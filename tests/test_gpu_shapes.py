@@ -178,6 +178,8 @@ def test_kernel_intervals_inside_graph_replays(torch):
     assert s["pair_timed_launches"] == s["score_launches"] > 0
     assert 0 < s["pair_busy_ms"] <= wall * 1.01 + 0.05
     assert s["pair_launch_ms"] >= s["pair_busy_ms"] * 0.999
+    # warp-time: positive, at most 24 resident one-warp CTAs per SM on average over the busy time
+    assert 0 < s["pair_warp_ms"] <= 24 * 148 * s["pair_busy_ms"] * 1.01
 
 
 def test_graph_cache_keeps_several_shapes(torch):
