@@ -196,6 +196,9 @@ static_assert(vsk::CELL_G % vsk::CELL_NSPLIT == 0, "the pair kernel assigns cell
 #ifndef VS_FILL_WARPS
 #define VS_FILL_WARPS 2048    // pair-kernel warps below which a scoring round uses KP = 1 chunks (launch shape)
 #endif
+#ifndef VS_TRIGGER_SPOTS
+#define VS_TRIGGER_SPOTS 0    // runs of at most this many spots: PDL early trigger (latency-bound)
+#endif
 #ifndef VS_DIRECT_GROUP_SPOTS
 #define VS_DIRECT_GROUP_SPOTS 16  // un-graphed runs: spots per stream group at least (small e2e 34 -> 24 ms / step)
 #endif
@@ -239,6 +242,7 @@ struct vs_ctx {
   int nsplit = 1;                        // canonical receptor-list splits (vs_score_params.list_splits)
   int force_kp = 0;                      // VS_SHAPE=kp (experiments)
   int direct_group_spots = VS_DIRECT_GROUP_SPOTS;  // spots per stream group at least, un-graphed runs
+  int trigger_spots = VS_TRIGGER_SPOTS;            // runs of at most this many spots use the PDL early trigger
   float4* d_ligx = nullptr;             // [n_lig] centred local coordinates, w = class
   float4* d_ligp = nullptr;             // [n_lig] es, c12, c6, donor
   int* d_lig_rank = nullptr;            // [n_lig] rank within the class
@@ -493,13 +497,14 @@ struct Group {
   CellArgs cplain, cls;                // scoring launches: plain (a whole population) and Improve (LS)
   int cplain_blocks = 0, cls_blocks = 0;
   bool in_b = false;  // the current population S sits in the second (B) buffer
+  int trig = 0;       // PDL early trigger for the group's chain (latency-bound runs)
 };
 
 // Improve (R16-R17): the best m of X by (score, index), then L fused
 // perturb -> score -> accept launches.
 vs_status improve_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, PoseRec* X, int g, Tracer* tr) {
   const int P = mp->population;
-  CK(launch_popsort(0, X, nullptr, nullptr, q.J, q.ns, P, m, q.st), "select launch");
+  CK(launch_popsort(0, X, nullptr, nullptr, q.J, q.ns, P, m, q.trig, q.st), "select launch");
   c->launches++;
   vs_status r = trace_idx(c, tr, q.st, VS_TRACE_SELECT, g, q.ns, m, q.J);
   if (r != VS_OK) return r;
@@ -517,7 +522,7 @@ vs_status improve_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, PoseR
 // Initialize(S): random population, scored, improved when f > 0, sorted.
 vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, Tracer* tr) {
   const int P = mp->population;
-  CK(launch_init(q.S, q.ns, P, q.seg, c->d_seed, c->T, q.st), "init launch");
+  CK(launch_init(q.S, q.ns, P, q.seg, c->d_seed, c->T, q.trig, q.st), "init launch");
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_INIT, 0, 0, q.ns, P, q.S);
   if (r != VS_OK) return r;
@@ -528,7 +533,7 @@ vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, Tra
   }
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, 0, 0, q.ns, P, q.S)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.S, 0, tr)) != VS_OK) return r;
-  CK(launch_popsort(1, q.S, nullptr, q.S2, nullptr, q.ns, P, m, q.st), "sort launch");
+  CK(launch_popsort(1, q.S, nullptr, q.S2, nullptr, q.ns, P, m, q.trig, q.st), "sort launch");
   c->launches++;
   std::swap(q.S, q.S2);
   q.in_b = !q.in_b;
@@ -538,7 +543,7 @@ vs_status gen_initialize(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, Tra
 // One pass of the while-loop body: Select + Combine, score, Improve, Include.
 vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, int g, Tracer* tr) {
   const int P = mp->population;
-  CK(launch_combine(q.S, q.C, q.ns, P, q.seg, c->d_seed, g, mp->p_mut, mp->mut_trans, mp->mut_rot, c->T, q.st),
+  CK(launch_combine(q.S, q.C, q.ns, P, q.seg, c->d_seed, g, mp->p_mut, mp->mut_trans, mp->mut_rot, c->T, q.trig, q.st),
      "combine launch");
   c->launches++;
   vs_status r = trace_poses(c, tr, q.st, VS_TRACE_COMBINED, g, 0, q.ns, P, q.C);
@@ -550,7 +555,7 @@ vs_status gen_step(vs_ctx* c, Group& q, const vs_mh_params* mp, int m, int g, Tr
   }
   if ((r = trace_poses(c, tr, q.st, VS_TRACE_SCORED, g, 0, q.ns, P, q.C)) != VS_OK) return r;
   if (mp->improve_frac > 0.0f && (r = improve_step(c, q, mp, m, q.C, g, tr)) != VS_OK) return r;
-  CK(launch_popsort(2, q.S, q.C, q.S2, nullptr, q.ns, P, m, q.st), "include launch");
+  CK(launch_popsort(2, q.S, q.C, q.S2, nullptr, q.ns, P, m, q.trig, q.st), "include launch");
   c->launches++;
   std::swap(q.S, q.S2);
   q.in_b = !q.in_b;
@@ -618,6 +623,9 @@ vs_status enqueue_body(vs_ctx* c, const Body& b, cudaStream_t st, Tracer* tr) {
       cl.K = mp->ls_neighbours;
       cl.ls_trans = mp->ls_trans;
       cl.ls_rot = mp->ls_rot;
+      // latency-bound runs (few spots): every chain kernel triggers its successor's launch at entry
+      q.trig = ns <= c->trigger_spots ? 1 : 0;
+      cp.trig = cl.trig = q.trig;
       q.cplain_blocks = q.ns * cp.nch_u * shp.nsg();
       q.cls_blocks = q.ns * cl.nch_u * shl.nsg();
     }
@@ -940,6 +948,7 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
   // launch-shape knobs for experiments (speed only; results never depend on them)
   if (const char* v = std::getenv("VS_FILL_WARPS")) c->fill_warps = std::max(1ll, std::atoll(v));
   if (const char* v = std::getenv("VS_DIRECT_GROUP_SPOTS")) c->direct_group_spots = std::max(1, std::atoi(v));
+  if (const char* v = std::getenv("VS_TRIGGER_SPOTS")) c->trigger_spots = std::atoi(v);
   if (const char* v = std::getenv("VS_SHAPE")) {  // "kp"
     const int kp = std::atoi(v);
     if (kp == 1 || kp == 2) c->force_kp = kp;

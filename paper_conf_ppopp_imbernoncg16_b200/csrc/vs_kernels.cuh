@@ -21,12 +21,16 @@ namespace vsk {
 #define VS_PDL_TRIGGER 0
 #endif
 
-__device__ __forceinline__ void pdl_enter() {
+// trig (runtime, per launch): also signal launch_dependents at entry, so the next kernel of the chain is scheduled
+// while this one runs and starts the instant it completes.  Used for latency-bound runs (few spots: the GPU has
+// idle slots for the waiting CTAs); for full runs the waiting CTAs would hold SM slots the other streams need.
+__device__ __forceinline__ void pdl_enter(int trig = 0) {
 #if VS_PDL
   asm volatile("griddepcontrol.wait;\n" ::: "memory");
 #if VS_PDL_TRIGGER
-  asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
+  trig = 1;
 #endif
+  if (trig) asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
 #endif
 }
 
@@ -133,6 +137,7 @@ struct CellArgs {
   unsigned long long* kt;
   const unsigned long long* kt_base;
   int kt_slot, kt_cap;
+  int trig;                  // PDL early trigger (latency-bound runs, pdl_enter)
 };
 constexpr int KT_WORDS = 3;  // per launch slot: ~start, end, sum of warp durations (ns)
 
@@ -157,13 +162,14 @@ cudaError_t launch_cell_scan(const int* counts, int n, int nn, int nh, int cn, i
                              int* chunk_prefix, int* cursor, cudaStream_t st);
 
 // launchers (return cudaError_t of the launch)
-cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, cudaStream_t st);
+cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, int trig,
+                        cudaStream_t st);
 cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, int g,
-                           float p_mut, float mut_trans, float mut_rot, float T, cudaStream_t st);
+                           float p_mut, float mut_trans, float mut_rot, float T, int trig, cudaStream_t st);
 // sort (score, index) per segment: mode 0: select best m indices -> J;
 // mode 1: sort S -> S_out; mode 2: include: best P of S ++ C -> S_out
 cudaError_t launch_popsort(int mode, const PoseRec* S, const PoseRec* C, PoseRec* S_out, int* J, int n_sel, int P,
-                           int m, cudaStream_t st);
+                           int m, int trig, cudaStream_t st);
 cudaError_t launch_best(const PoseRec* S, int n_sel, int P, float* best_pose, float* best_score, cudaStream_t st);
 cudaError_t launch_build_lists(const float4* rec, const float4* rprm, int n_rec, const float4* spot_c, int n_spots,
                                float reach2, const int* off, int* len, RecAtom* lists, int count_only,

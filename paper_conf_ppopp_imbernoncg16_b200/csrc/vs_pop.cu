@@ -12,8 +12,8 @@
 
 namespace vsk {
 
-__global__ void init_kernel(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T) {
-  pdl_enter();  // PDL: predecessor complete and visible (vs_kernels.cuh)
+__global__ void init_kernel(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, int trig) {
+  pdl_enter(trig);  // PDL: predecessor complete and visible (vs_kernels.cuh)
   const uint64_t seed = *seedp;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= n_sel * P) return;
@@ -29,8 +29,8 @@ __global__ void init_kernel(PoseRec* S, int n_sel, int P, const int* seg_spot, c
 // child j of generation g from the sorted population S (rank = index)
 __global__ void combine_kernel(const PoseRec* __restrict__ S, PoseRec* __restrict__ C, int n_sel, int P,
                                const int* seg_spot, const uint64_t* seedp, int g, float p_mut, float mut_trans,
-                               float mut_rot, float T) {
-  pdl_enter();  // PDL: predecessor complete and visible (vs_kernels.cuh)
+                               float mut_rot, float T, int trig) {
+  pdl_enter(trig);  // PDL: predecessor complete and visible (vs_kernels.cuh)
   const uint64_t seed = *seedp;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= n_sel * P) return;
@@ -77,8 +77,8 @@ __device__ __forceinline__ uint64_t pkey(float score, uint32_t idx) {
 // One CTA per spot.  mode 0: J = best m of S by (score, index);
 // mode 1: S_out = S sorted; mode 2: S_out = best P of S ++ C (S first on ties).
 __global__ void popsort_kernel(int mode, const PoseRec* __restrict__ S, const PoseRec* __restrict__ C,
-                               PoseRec* __restrict__ S_out, int* __restrict__ J, int P, int m, int N) {
-  pdl_enter();  // PDL: predecessor complete and visible (vs_kernels.cuh)
+                               PoseRec* __restrict__ S_out, int* __restrict__ J, int P, int m, int N, int trig) {
+  pdl_enter(trig);  // PDL: predecessor complete and visible (vs_kernels.cuh)
   extern __shared__ uint64_t keys[];
   const int k = blockIdx.x;
   const int count = mode == 2 ? 2 * P : P;
@@ -214,24 +214,25 @@ __global__ void scatter_kernel(int64_t n, const int32_t* spot, const float* q, c
 // ---------------------------------------------------------------- launchers
 static inline int nblk(int64_t n, int b) { return (int)((n + b - 1) / b); }
 
-cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, cudaStream_t st) {
-  return launch_chain(init_kernel, nblk((int64_t)n_sel * P, 128), 128, 0, st, S, n_sel, P, seg_spot, seedp, T);
+cudaError_t launch_init(PoseRec* S, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, float T, int trig,
+                        cudaStream_t st) {
+  return launch_chain(init_kernel, nblk((int64_t)n_sel * P, 128), 128, 0, st, S, n_sel, P, seg_spot, seedp, T, trig);
 }
 
 cudaError_t launch_combine(const PoseRec* S, PoseRec* C, int n_sel, int P, const int* seg_spot, const uint64_t* seedp, int g,
-                           float p_mut, float mut_trans, float mut_rot, float T, cudaStream_t st) {
+                           float p_mut, float mut_trans, float mut_rot, float T, int trig, cudaStream_t st) {
   return launch_chain(combine_kernel, nblk((int64_t)n_sel * P, 128), 128, 0, st, S, C, n_sel, P, seg_spot, seedp, g, p_mut,
-                      mut_trans, mut_rot, T);
+                      mut_trans, mut_rot, T, trig);
 }
 
 cudaError_t launch_popsort(int mode, const PoseRec* S, const PoseRec* C, PoseRec* S_out, int* J, int n_sel, int P,
-                           int m, cudaStream_t st) {
+                           int m, int trig, cudaStream_t st) {
   const int count = mode == 2 ? 2 * P : P;
   int N = 2;
   while (N < count) N <<= 1;
   const int threads = min(1024, max(32, N / 2));
   const size_t smem = sizeof(uint64_t) * N;
-  return launch_chain(popsort_kernel, n_sel, threads, smem, st, mode, S, C, S_out, J, P, m, N);
+  return launch_chain(popsort_kernel, n_sel, threads, smem, st, mode, S, C, S_out, J, P, m, N, trig);
 }
 
 cudaError_t launch_best(const PoseRec* S, int n_sel, int P, float* best_pose, float* best_score, cudaStream_t st) {
