@@ -177,6 +177,15 @@ VS_API void vs_destroy(vs_ctx* c); /* NULL-safe; synchronises the ctx's device w
  * cached blocks of `cuda_device` (< 0: of every device) to the driver; live contexts keep theirs.  Thread-safe.
  * Errors: VS_ERR_INVALID_ARGUMENT (no such device). */
 VS_API vs_status vs_release_cached_memory(int32_t cuda_device);
+
+/* Environment variables read at vs_create (speed experiments only: no result depends on them):
+ *   VS_GRAPHS=0             never capture CUDA graphs (plain launches, e.g. for profilers)
+ *   VS_FILL_WARPS=n         scoring rounds with fewer pair-kernel warps than n use KP = 1 chunks (default 2048)
+ *   VS_SHAPE=1|2            force the chunk shape KP
+ *   VS_DIRECT_GROUP_SPOTS=n spots per stream group at least in un-graphed runs (default 16)
+ *   VS_CELL_MERGE=0|1       one item class for every launch (default 0; KP = 1 launches merge anyway)
+ *   VS_TRIGGER_SPOTS=n      runs of at most n spots use the PDL early trigger (default 0: off)
+ *   VS_POOL_CACHE_MB=n      device memory cache cap (above) */
 VS_API const char* vs_last_error(void);
 VS_API int vs_abi_version(void);
 
