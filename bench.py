@@ -71,7 +71,8 @@ def parse(argv=None):
     ap.add_argument("--scaling", choices=["strong", "replicas"], default="strong")
     ap.add_argument("--schedule", choices=["queue", "static", "warmup"], default="queue")
     ap.add_argument("--chunks-per-rank", type=int, default=1, help="queue: chunks = ranks x this")
-    ap.add_argument("--slots", type=int, default=1, help="queue: chunks in flight per rank (one context each)")
+    ap.add_argument("--slots", type=int, default=None,
+                    help="queue: chunks in flight per rank, one context / stream each (default 1; sweep 2)")
     ap.add_argument("--list-splits", type=int, default=-1,
                     help="vs_score_params.list_splits (-1: by the spots per rank, 0: by the context)")
     ap.add_argument("--hetero", default="", help="injected heterogeneity 'rank:factor,...' (each chunk run factor x)")
@@ -174,6 +175,22 @@ def ncu_traffic(config: str):
         except (OSError, ValueError):
             pass
     return None
+
+
+def union_ms(iv) -> float:
+    """Length in ms of the union of [start, end) intervals given in ns ([n, 2])."""
+    if len(iv) == 0:
+        return 0.0
+    iv = iv[np.argsort(iv[:, 0], kind="stable")]
+    tot, cs, ce = 0, int(iv[0, 0]), int(iv[0, 1])
+    for a, b in iv[1:]:
+        a, b = int(a), int(b)
+        if a > ce:
+            tot += ce - cs
+            cs, ce = a, b
+        elif b > ce:
+            ce = b
+    return (tot + ce - cs) * 1e-6
 
 
 def hetero_factor(spec: str, rank: int) -> int:
@@ -383,6 +400,8 @@ def main():
     prob = synth.make_problem(args.config)
     cfg = prob.cfg
     sweep = cfg.n_ligands > 1
+    if args.slots is None:   # two ligands in flight: the sweep's P 64 runs are partly latency-bound (r02_notes.md)
+        args.slots = 2 if sweep else 1
     G = cfg.generations if args.generations is None else args.generations
     cutoff = 12.0 if args.mode == "cutoff" else 0.0
     n_spots = cfg.n_spots
@@ -515,9 +534,14 @@ def main():
     ms_rank = e0.elapsed_time(e1)
     work_ctx = list(scr.ctx.values()) if sweep else runner.ctx
     st = {}
+    ivs = []
     for c in work_ctx:
         for k, v in c.stats().items():
             st[k] = st.get(k, 0) + v
+        ivs.append(c.pair_intervals())
+    # contexts (slots, ligands) run concurrently: the pair kernel's busy time is the union of all their launch
+    # intervals on the device clock, not the sum of the per-context unions
+    st["pair_busy_ms"] = union_ms(np.concatenate(ivs)) if ivs else 0.0
     if sweep:
         scr.set_timing(0)
     else:

@@ -223,6 +223,11 @@ VS_API vs_status vs_set_timing(vs_ctx* c, int flags);
 /* Synchronises the ctx's device and returns counters since the last reset. */
 VS_API vs_status vs_get_stats(vs_ctx* c, vs_stats* out);
 VS_API vs_status vs_reset_stats(vs_ctx* c);
+/* VS_TIMING_KERNEL: the pair kernel's launch intervals since the last reset as (start, end) device globaltimer ns
+ * pairs into out[cap][2] (one clock per device, so the intervals of several contexts can be merged: their union is
+ * the time some pair kernel ran).  Returns the number recorded (only min(n, cap) written; cap 0 with out NULL
+ * queries n), 0 if kernel timing was never enabled, -1 on error (vs_last_error). */
+VS_API int64_t vs_pair_intervals(vs_ctx* c, uint64_t* out, int64_t cap);
 /* Per-spot receptor list lengths (cutoff mode) or n_rec (all pairs). */
 VS_API vs_status vs_list_lengths(vs_ctx* c, int32_t* out /*[n_spots]*/);
 

@@ -1411,6 +1411,33 @@ vs_status vs_reset_stats(vs_ctx* c) {
   return VS_OK;
 }
 
+int64_t vs_pair_intervals(vs_ctx* c, uint64_t* out, int64_t cap) {
+  if (!c || cap < 0 || (cap > 0 && !out)) {
+    set_err(VS_ERR_INVALID_ARGUMENT, "bad arguments");
+    return -1;
+  }
+  if (c->poisoned || !c->d_kt) return 0;
+  DeviceGuard guard(c->dev);
+  if (cudaDeviceSynchronize() != cudaSuccess) return -1;
+  unsigned long long nslot = 0;
+  if (cudaMemcpy(&nslot, c->d_kt_base, sizeof(nslot), cudaMemcpyDeviceToHost) != cudaSuccess) return -1;
+  nslot = std::min<unsigned long long>(nslot, VS_KT_CAP);
+  std::vector<unsigned long long> kt(KT_WORDS * nslot);
+  if (nslot && cudaMemcpy(kt.data(), c->d_kt, sizeof(unsigned long long) * KT_WORDS * nslot, cudaMemcpyDeviceToHost) !=
+                   cudaSuccess)
+    return -1;
+  int64_t n = 0;
+  for (unsigned long long i = 0; i < nslot; ++i)
+    if (kt[KT_WORDS * i] && kt[KT_WORDS * i + 1] && kt[KT_WORDS * i + 1] >= ~kt[KT_WORDS * i]) {
+      if (n < cap) {
+        out[2 * n] = ~kt[KT_WORDS * i];
+        out[2 * n + 1] = kt[KT_WORDS * i + 1];
+      }
+      ++n;
+    }
+  return n;
+}
+
 vs_status vs_list_lengths(vs_ctx* c, int32_t* out) {
   if (!c || !out) return set_err(VS_ERR_INVALID_ARGUMENT, "NULL argument");
   std::memcpy(out, c->h_list_len.data(), sizeof(int32_t) * c->n_spots);

@@ -23,7 +23,7 @@ TRACE_INIT, TRACE_SCORED, TRACE_SELECT, TRACE_LS, TRACE_SORTED, TRACE_COMBINED, 
 EXPORTS = ["vs_score_params_default", "vs_mh_preset", "vs_create", "vs_score_poses", "vs_score_poses_device",
            "vs_run", "vs_run_async", "vs_destroy", "vs_last_error", "vs_abi_version", "vs_set_timing",
            "vs_get_stats", "vs_reset_stats", "vs_list_lengths", "vs_run_trace", "vs_debug_philox",
-           "vs_release_cached_memory"]
+           "vs_release_cached_memory", "vs_pair_intervals"]
 
 
 def release_cached_memory(device: int = -1) -> None:
@@ -113,6 +113,8 @@ def load(build_if_stale: bool = True):
     L.vs_get_stats.argtypes = [vp, C.POINTER(Stats)]
     L.vs_reset_stats.argtypes = [vp]
     L.vs_list_lengths.argtypes = [vp, i32p]
+    L.vs_pair_intervals.argtypes = [vp, C.POINTER(C.c_uint64), C.c_int64]
+    L.vs_pair_intervals.restype = C.c_int64
     L.vs_debug_philox.argtypes = [C.c_int64, u32p, u32p, u32p]
     _lib = L
     return L
@@ -269,6 +271,18 @@ class Context:
 
     def reset_stats(self):
         _check(load().vs_reset_stats(self.h))
+
+    def pair_intervals(self) -> np.ndarray:
+        """[n, 2] uint64 (start, end) device-globaltimer ns of the pair kernel's launches (VS_TIMING_KERNEL)."""
+        L = load()
+        n = L.vs_pair_intervals(self.h, None, 0)
+        if n < 0:
+            raise VSError(ERR_CUDA, L.vs_last_error().decode())
+        out = np.zeros((max(n, 1), 2), np.uint64)
+        n = L.vs_pair_intervals(self.h, out.ctypes.data_as(C.POINTER(C.c_uint64)), len(out))
+        if n < 0:
+            raise VSError(ERR_CUDA, L.vs_last_error().decode())
+        return out[:min(n, len(out))]
 
     def list_lengths(self) -> np.ndarray:
         o = np.zeros(self.n_spots, np.int32)

@@ -90,4 +90,7 @@ def test_hetero_and_splits_helpers():
     import bench
     assert bench.hetero_factor("0:2,3:4", 0) == 2 and bench.hetero_factor("0:2,3:4", 3) == 4
     assert bench.hetero_factor("", 1) == 1
+    import numpy as np
+    iv = np.array([[20, 30], [0, 10], [5, 12], [25, 26], [12, 13]], np.uint64) * 1000000
+    assert bench.union_ms(iv) == 23.0 and bench.union_ms(np.zeros((0, 2), np.uint64)) == 0.0
     assert bench.auto_splits(500) == 1 and bench.auto_splits(250) == 1 and bench.auto_splits(125) == 2 and bench.auto_splits(63) == 4

@@ -180,6 +180,12 @@ def test_kernel_intervals_inside_graph_replays(torch):
     assert s["pair_launch_ms"] >= s["pair_busy_ms"] * 0.999
     # warp-time: positive, at most 24 resident one-warp CTAs per SM on average over the busy time
     assert 0 < s["pair_warp_ms"] <= 24 * 148 * s["pair_busy_ms"] * 1.01
+    # the raw intervals (vs_pair_intervals): as many as timed launches, their sum and union are the stats'
+    iv = g.pair_intervals().astype(np.int64)
+    assert len(iv) == s["pair_timed_launches"] and np.all(iv[:, 1] >= iv[:, 0])
+    assert abs((iv[:, 1] - iv[:, 0]).sum() * 1e-6 - s["pair_launch_ms"]) < 1e-3
+    import bench
+    assert abs(bench.union_ms(iv) - s["pair_busy_ms"]) < 1e-3
 
 
 def test_graph_cache_keeps_several_shapes(torch):
