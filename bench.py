@@ -454,6 +454,8 @@ def main():
                 ids = np.arange(wn, dtype=np.int32)
                 runner.ctx[0].run_async(mpw, args.seed, ids, wp, ws, main_stream)   # untimed: lazy set-up
                 torch.cuda.synchronize(dev)
+                if world > 1:
+                    dist.barrier()  # no rank times its warm-up while another still does its lazy set-up
                 t0 = time.perf_counter()
                 for _ in range(rep):
                     runner.ctx[0].run_async(mpw, args.seed, ids, wp, ws, main_stream)

@@ -144,3 +144,24 @@ def test_scores_independent_of_batch_composition(gpu, medium):
     np.testing.assert_array_equal(g.score_poses(spot[s0], q[s0], t[s0]), full[s0])
     dup = np.concatenate([np.arange(3000), np.arange(3000)])
     np.testing.assert_array_equal(g.score_poses(spot[dup], q[dup], t[dup]), full[dup])
+
+
+@pytest.mark.parametrize("S", [1, 4])
+@pytest.mark.parametrize("cutoff", [12.0, 0.0])
+@pytest.mark.parametrize("roles", ["none", "all"])
+def test_receptor_role_extremes(gpu, oracle_mod, roles, cutoff, S):
+    """Receptors at the two extremes of the H-bond term (R5): no donor / acceptor atom at all (every H-bond sum is 0)
+    and only donor / acceptor atoms (every pair of an H-bond ligand atom carries H-bond terms), with an H-bond-rich
+    ligand, in both modes and list splits: within the tolerance of the oracle."""
+    prob = synth.make_custom(2500, 23, 6, seed=21)
+    rng = np.random.default_rng(2)
+    kinds = [synth.T_C, synth.T_H] if roles == "none" else [synth.T_N, synth.T_O, synth.T_HD]
+    prob.rec.type[:] = rng.choice(kinds, size=len(prob.rec.type)).astype(np.int32)
+    prob.lig.type[:] = rng.choice([synth.T_N, synth.T_O, synth.T_HD, synth.T_C, synth.T_H],
+                                  size=len(prob.lig.type)).astype(np.int32)
+    spot, q, t = synth.make_poses(1500, prob.cfg.n_spots, 3.0, seed=3)
+    t[:500] *= 0.3
+    got = vs.Context.from_problem(prob, vs.score_params(cutoff=cutoff, list_splits=S)).score_poses(spot, q, t)
+    o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params(cutoff=cutoff))
+    idx = np.arange(0, len(spot), 7)
+    assert_scores(got[idx], o.score(spot[idx], q[idx], t[idx]), f"receptor roles {roles}")
