@@ -22,6 +22,8 @@ def main():
     ap.add_argument("--generations", type=int, default=1)
     ap.add_argument("--score-poses", type=int, default=0, help="also score N random poses via vs_score_poses")
     ap.add_argument("--graph", action="store_true", help="direct run, captured run, then one graph replay")
+    ap.add_argument("--replay-only", action="store_true",
+                    help="with --graph: cudaProfilerStart/Stop around the replay (ncu --profile-from-start off)")
     args = ap.parse_args()
     import torch
     from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
@@ -32,7 +34,12 @@ def main():
     if args.graph:
         g.run(mp, 42)          # captured
         torch.cuda.synchronize()
+        if args.replay_only:   # ncu --profile-from-start off: only the replayed graph is profiled
+            torch.cuda.profiler.start()
         g.run(mp, 42)          # replayed
+        torch.cuda.synchronize()
+        if args.replay_only:
+            torch.cuda.profiler.stop()
     if args.score_poses:
         spot, q, t = synth.make_poses(args.score_poses, prob.cfg.n_spots, 3.0, seed=1)
         g.score_poses(spot, q, t)
