@@ -22,7 +22,10 @@ case $what in
    unset VS_BENCH_BACKEND ;;
  ll) VS_GRAPHS=0 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_medium_g10.csv python tools/prof_run.py --generations 10 > $O/ll.log 2>&1 ;;
  ncu) VS_GRAPHS=0 timeout 900 ncu --set full --clock-control none --import-source on -k regex:cell_pair_kernel -c 2 -f -o $O/pair python tools/prof_run.py --generations 1 > $O/ncu_pair.log 2>&1 ;;
- graph) timeout 900 ncu --graph-profiling graph --clock-control none --metrics gpu__time_duration.sum,sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_elapsed,sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_elapsed,smsp__issue_active.avg.pct_of_peak_sustained_elapsed,sm__warps_active.avg.pct_of_peak_sustained_elapsed,sm__inst_executed_pipe_xu.avg.pct_of_peak_sustained_elapsed,sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_elapsed,dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum,sm__cycles_elapsed.avg.per_second --csv --log-file $O/graph_medium_g10.csv python tools/prof_run.py --generations 10 --graph > $O/graph.log 2>&1 ;;
+ graph) timeout 900 ncu --graph-profiling graph --profile-from-start off --clock-control none --metrics gpu__time_duration.sum,sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_elapsed,sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_elapsed,smsp__issue_active.avg.pct_of_peak_sustained_elapsed,sm__warps_active.avg.pct_of_peak_sustained_elapsed,sm__inst_executed_pipe_xu.avg.pct_of_peak_sustained_elapsed,sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_elapsed,dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum,sm__cycles_elapsed.avg.per_second,smsp__average_warps_issue_stalled_wait_per_issue_active.ratio,smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio,smsp__average_warps_issue_stalled_math_pipe_throttle_per_issue_active.ratio,smsp__average_warps_issue_stalled_not_selected_per_issue_active.ratio,smsp__average_warps_issue_stalled_no_instruction_per_issue_active.ratio --csv --log-file $O/graph_medium_g10.csv python tools/prof_run.py --generations 10 --graph --replay-only > $O/graph.log 2>&1 ;;
+ ref) $B --impl reference > $O/bench_reference.jsonl 2> $O/bench_reference.err ;;
+ tests) timeout 1500 python -m pytest tests -x -q -m gpu > $O/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $O/pytest_gpu.log ;;
+ smoke) python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log ;;
 esac
 done
 ls -la $O
