@@ -674,7 +674,7 @@ def main():
         for i in range(n_e2e):
             if sweep:
                 q = vdist.ChunkQueue(store, f"e{i}", len(units))
-                ctxs = {}
+                ctxs = {}  # a rank closes a ligand's context after the ligand's last unit (device memory back to the cache)
                 while (u := q.claim()) is not None:
                     li, a, b = units[u]
                     ta = time.perf_counter()
@@ -685,8 +685,14 @@ def main():
                     ctxs[li].run(mp, screen.ligand_seed(args.seed, li), np.arange(a, b, dtype=np.int32))
                     h2d += 4 * (b - a)
                     d2h += 32 * (b - a)
+                    tc = time.perf_counter()
                     parts_ms["create"] += 1e3 * (tb - ta)
-                    parts_ms["run"] += 1e3 * (time.perf_counter() - tb)
+                    parts_ms["run"] += 1e3 * (tc - tb)
+                    # units are claimed in order (ligands by decreasing size, then chunks): once the queue has moved
+                    # past a ligand's last unit no rank can claim more of it
+                    if all(units[v][0] != li for v in range(u + 1, len(units))):
+                        ctxs.pop(li).close()
+                        parts_ms["destroy"] += 1e3 * (time.perf_counter() - tc)
                 tc = time.perf_counter()
                 for c in ctxs.values():
                     c.close()
