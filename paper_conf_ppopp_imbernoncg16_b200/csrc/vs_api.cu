@@ -235,6 +235,9 @@ struct vs_ctx {
   float4* d_shift = nullptr;
   int* d_iota = nullptr;
   unsigned long long* d_counters = nullptr;  // [0] pairs evaluated, [1] poses, [2] workload pairs, [3] within rc
+  // vs_run's scored poses and workload pairs, counted on the host from the run's parameters (K3 counts them on the
+  // device only for vs_score_poses: a burst of same-address atomics from every K3 CTA cost 0.4 % of a medium step)
+  unsigned long long host_poses = 0, host_pairs = 0;
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
   uint16_t* d_cells = nullptr;          // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
   float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
@@ -681,6 +684,15 @@ vs_status run_impl(vs_ctx* c, const vs_mh_params* mp, uint64_t seed, int32_t n_s
     CK(c->buf[B_PBUF].ensure(sizeof(PoseRec) * (size_t)ns * maxpose), "alloc");
     CK(c->buf[B_ITEMS].ensure(sizeof(float4) * (size_t)ns * maxpose * c->n_lig), "alloc");
     CK(c->buf[B_E].ensure(sizeof(double) * (size_t)ns * c->n_lig * emax), "alloc");
+  }
+  {  // every spot scores (G + 1) x (P + L m K) poses (init / Combine rounds, Improve proposals), n_lig x list pairs each
+    const unsigned long long per =
+        (unsigned long long)(mp->generations + 1) *
+        ((unsigned long long)P + (mp->improve_frac > 0.0f ? (unsigned long long)mp->ls_steps * m * mp->ls_neighbours : 0ull));
+    unsigned long long lsum = 0;
+    for (int k = 0; k < ns; ++k) lsum += (unsigned long long)c->h_list_len[spot_ids ? spot_ids[k] : k];
+    c->host_poses += per * (unsigned long long)ns;
+    c->host_pairs += per * (unsigned long long)c->n_lig * lsum;
   }
   int* seg = (int*)c->buf[B_SEG].p;
   if (spot_ids)
@@ -1345,6 +1357,8 @@ vs_status vs_get_stats(vs_ctx* c, vs_stats* o) {
   if (s != VS_OK) return s;
   unsigned long long h[4];
   CK(cudaMemcpy(h, c->d_counters, sizeof(h), cudaMemcpyDeviceToHost), "D2H counters");
+  h[1] += c->host_poses;
+  h[2] += c->host_pairs;
   o->pairs_within = c->all_pairs ? h[2] : h[3];  // all-pairs mode: every pair is within
   o->pair_busy_ms = o->pair_launch_ms = o->pair_warp_ms = 0.0;
   o->pair_timed_launches = 0;
@@ -1400,6 +1414,7 @@ vs_status vs_reset_stats(vs_ctx* c) {
   DeviceGuard guard(c->dev);
   CK(cudaDeviceSynchronize(), "sync");
   CK(cudaMemset(c->d_counters, 0, sizeof(unsigned long long) * 4), "memset");
+  c->host_poses = c->host_pairs = 0;
   if (c->d_kt) {
     CK(cudaMemset(c->d_kt, 0, sizeof(unsigned long long) * KT_WORDS * (size_t)VS_KT_CAP), "memset");
     CK(cudaMemset(c->d_kt_base, 0, sizeof(unsigned long long)), "memset");

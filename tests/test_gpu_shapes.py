@@ -247,3 +247,25 @@ def test_no_hbond_ligand_kp1(torch, oracle_mod):
     o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params())
     r = o.score(spot[:60], q[:60], t[:60])
     assert np.all(np.abs(res[0][:60] - r) <= np.maximum(1e-4 * np.abs(r), 1e-3))
+
+
+@pytest.mark.parametrize("preset,K", [(3, 1), (1, 1), (4, 3)])
+def test_run_stats_count_scored_poses_and_pairs(torch, preset, K):
+    """vs_run's `poses_scored` and `pairs` (workload pairs: n_lig x list length of the pose's spot per scored pose):
+    every spot scores (G + 1) x (P + L m K) poses -- the initial / offspring rounds and Improve's proposals, m =
+    round(f P) (S§8(c) R17)."""
+    prob = synth.make_problem("small")
+    g = vs.Context.from_problem(prob, vs.score_params())
+    mp = vs.mh_preset(preset, population=32, generations=3 if preset != 4 else 0, ls_neighbours=K)
+    ids = np.array([3, 0, 17, 5, 3], dtype=np.int32)[:4]
+    g.reset_stats()
+    g.run(mp, 5, ids)
+    g.run(mp, 6)
+    st = g.stats()
+    m = max(1, min(mp.population, int(np.floor(float(np.float32(mp.improve_frac)) * mp.population + 0.5)))) \
+        if mp.improve_frac > 0 else 0
+    per = (mp.generations + 1) * (mp.population + (mp.ls_steps * m * K if mp.improve_frac > 0 else 0))
+    L = g.list_lengths()
+    n_all = prob.cfg.n_spots
+    assert st["poses_scored"] == per * (len(ids) + n_all)
+    assert st["pairs"] == per * prob.cfg.n_lig * (int(sum(int(L[s]) for s in ids)) + int(sum(int(x) for x in L)))

@@ -21,6 +21,8 @@ def main():
     ap.add_argument("--preset", type=int, default=3)
     ap.add_argument("--generations", type=int, default=1)
     ap.add_argument("--score-poses", type=int, default=0, help="also score N random poses via vs_score_poses")
+    ap.add_argument("--spots", type=int, default=0, help="run only the first N spots (0: all)")
+    ap.add_argument("--splits", type=int, default=0, help="vs_score_params.list_splits (0: the context default)")
     ap.add_argument("--graph", action="store_true", help="direct run, captured run, then one graph replay")
     ap.add_argument("--replay-only", action="store_true",
                     help="with --graph: cudaProfilerStart/Stop around the replay (ncu --profile-from-start off)")
@@ -28,15 +30,17 @@ def main():
     import torch
     from paper_conf_ppopp_imbernoncg16_b200 import synth, vs
     prob = synth.make_problem(args.config)
-    g = vs.Context.from_problem(prob, vs.score_params(), device=0)
+    g = vs.Context.from_problem(prob, vs.score_params(**({"list_splits": args.splits} if args.splits else {})), device=0)
     mp = vs.mh_preset(args.preset, population=prob.cfg.population, generations=args.generations)
-    g.run(mp, 42)
+    import numpy as np
+    ids = np.arange(args.spots, dtype=np.int32) if args.spots else None
+    g.run(mp, 42, ids)
     if args.graph:
-        g.run(mp, 42)          # captured
+        g.run(mp, 42, ids)     # captured
         torch.cuda.synchronize()
         if args.replay_only:   # ncu --profile-from-start off: only the replayed graph is profiled
             torch.cuda.profiler.start()
-        g.run(mp, 42)          # replayed
+        g.run(mp, 42, ids)     # replayed
         torch.cuda.synchronize()
         if args.replay_only:
             torch.cuda.profiler.stop()
