@@ -183,7 +183,18 @@ struct DevBuf {
 #define VS_NSUB 12
 #endif
 constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
-static_assert(vsk::CELL_G % vsk::CELL_NSPLIT == 0, "the pair kernel assigns cell rows to splits by cy mod NSPLIT");
+// cells per axis of the per-spot list grid: 16 for contexts with 1 or 2 list splits (throughput-bound runs: fewer,
+// longer row runs), 20 with 4 splits (latency-bound runs: each split warp streams fewer atoms).  Medium, ms: S 1,
+// 500 spots: G 24 / 20 / 16 / 12 465.3 / 464.2 / 459.9 / 462.4; S 2, 125 spots 129.0 / 128.1 / 127.3; S 4, 63
+// spots 78.0 / 77.1 / 78.5; small (S 4) 17.9 / 17.57 / 18.2; large 500 spots (S 1) 1260 / 1256 / 1247
+// (profiles/r02_notes.md).  S must divide G (the pair kernel assigns cell rows to splits by cy mod S).
+int cell_grid(int nsplit) {
+  const int g = VS_CELL_G > 0 ? VS_CELL_G : (nsplit >= 4 ? 20 : 16);
+  return g;
+}
+static_assert(vsk::CELL_GMAX % vsk::CELL_NSPLIT == 0 && 20 % vsk::CELL_NSPLIT == 0 && 16 % vsk::CELL_NSPLIT == 0,
+              "the pair kernel assigns cell rows to splits by cy mod S");
+static_assert(VS_CELL_G <= vsk::CELL_GMAX && VS_CELL_G % vsk::CELL_NSPLIT == 0, "VS_CELL_G");
 #ifndef VS_GROUP_SPOTS
 #define VS_GROUP_SPOTS 8    // spots per stream group at least
 #endif
@@ -239,7 +250,8 @@ struct vs_ctx {
   // device only for vs_score_poses: a burst of same-address atomics from every K3 CTA cost 0.4 % of a medium step)
   unsigned long long host_poses = 0, host_pairs = 0;
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
-  uint16_t* d_cells = nullptr;          // cutoff mode: [n_spots][CELL_G3 + 1] cell starts of the cell-sorted lists
+  uint16_t* d_cells = nullptr;          // cutoff mode: [n_spots][cg^3 + 1] cell starts of the cell-sorted lists
+  int cell_g = 16;                      // cells per axis of the list grid (cell_grid)
   float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
   long long fill_warps = VS_FILL_WARPS;  // launch shape target (speed only)
   int nsplit = 1;                        // canonical receptor-list splits (vs_score_params.list_splits)
@@ -395,6 +407,7 @@ CellArgs cell_base(vs_ctx* c) {
   a.cR = c->cR;
   a.ch = c->ch;
   a.cinv_h = c->cinv_h;
+  a.cg = c->cell_g;
   a.ligx = c->d_ligx;
   a.ligp = c->d_ligp;
   a.lig_rank = c->d_lig_rank;
@@ -1140,11 +1153,13 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     RecAtom* sorted = nullptr;
     CKT(pool::alloc(&sorted, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
     c->cR = (float)reach + 0.01f;
-    c->ch = 2.0f * c->cR / (float)CELL_G;
-    c->cinv_h = (float)CELL_G / (2.0f * c->cR);
-    CKT(pool::alloc(&c->d_cells, sizeof(uint16_t) * (size_t)n_spots * (CELL_G3 + 1)), "alloc cell tables");
-    cudaError_t es = launch_cell_sort(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_cells, c->cR,
-                                      c->cinv_h, c->stream);
+    c->cell_g = cell_grid(c->nsplit);
+    const int G = c->cell_g;
+    c->ch = 2.0f * c->cR / (float)G;
+    c->cinv_h = (float)G / (2.0f * c->cR);
+    CKT(pool::alloc(&c->d_cells, sizeof(uint16_t) * (size_t)n_spots * ((size_t)G * G * G + 1)), "alloc cell tables");
+    cudaError_t es = launch_cell_sort(c->d_lists, sorted, c->d_list_off, c->d_list_len, n_spots, c->d_cells, G,
+                                      c->cR, c->cinv_h, c->stream);
     if (es == cudaSuccess) es = cudaStreamSynchronize(c->stream);
     pool::release(c->d_lists);
     c->d_lists = sorted;

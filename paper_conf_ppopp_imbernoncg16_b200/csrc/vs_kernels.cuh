@@ -64,13 +64,12 @@ enum ScoreMode : int { MODE_PLAIN = 0, MODE_LS = 1 };
 #define VS_CELL_MERGE 0  // 1: every ligand atom in class 1 (one item order, all slot pairs H-bond pairs)
 #endif
 #ifndef VS_CELL_G
-#define VS_CELL_G 24
+#define VS_CELL_G 0  // 0: cells per axis chosen per context from its list splits (vs_api.cu cell_grid); > 0 forces it
 #endif
 #ifndef VS_CELL_EXACTX
 #define VS_CELL_EXACTX 0  // exact-x trim of row runs: redundant with the per-pair atom test (VS_CELL_PPCULL), measured 1.4 % slower
 #endif
-constexpr int CELL_G = VS_CELL_G;                  // list grid per spot: G^3 cells over [-R, R]^3 (G <= 64)
-constexpr int CELL_G3 = CELL_G * CELL_G * CELL_G;
+constexpr int CELL_GMAX = 24;                      // largest list grid per spot: G^3 cells over [-R, R]^3, G <= 24
 constexpr int CELL_SORT_MAX = 16384;               // longest list cell-sorted in shared memory (128 KB keys)
 constexpr int CELL_KP = 2;                         // packed float2 item pairs per lane of the default pair kernel
 constexpr int CH_ITEMS = 2 * CELL_KP * 32;         // items per chunk (one warp) of the default pair kernel
@@ -79,18 +78,19 @@ constexpr int CELL_NSPLIT = 4;                     // most canonical receptor-li
 #define VS_CELL_BATCH 64
 #endif
 constexpr int CELL_BATCH = VS_CELL_BATCH;          // receptor atoms per staging buffer (2 per lane per 64)
-constexpr int CELL_MAXRUN = CELL_G * CELL_G;       // one run per cell row at most
+constexpr int CELL_MAXRUN = CELL_GMAX * CELL_GMAX; // one run per cell row at most
 constexpr int MORTON_BITS = 4;                     // item sort grid: 16^3 cells over the spot region
 constexpr int MORTON_BINS = 1 << (3 * MORTON_BITS);
 
 struct CellArgs {
-  // receptor lists (per spot) and the cell start table [n_spots][CELL_G3 + 1] (uint16 list positions; a
+  // receptor lists (per spot) and the cell start table [n_spots][cg^3 + 1] (uint16 list positions; a
   // cell-sorted list has <= CELL_SORT_MAX < 2^16 atoms; cells[s][0] == 0xFFFF: not cell-sorted -> streamed whole)
   const RecAtom* lists;
   const int* list_off;
   const int* list_len;
   const uint16_t* cells;
   float cR, ch, cinv_h;      // grid half-width (A), cell edge, 1 / edge
+  int cg;                    // cells per axis of the list grid (a context property; S divides it)
   // ligand (input order)
   const float4* ligx;        // local x, y, z (centred), w = class (0: class 0; 1: class 1, donor / acceptor; 2: class 1, no role)
   const float4* ligp;        // es_i, c12_i, c6_i, donor_i
@@ -154,7 +154,7 @@ __host__ __device__ inline int cell_chunks(int seg_n, int nn, int nh, int cap, i
 }
 
 cudaError_t launch_cell_sort(const RecAtom* lists, RecAtom* out, const int* off, const int* len, int n_spots, uint16_t* cells,
-                             float R, float inv_h, cudaStream_t st);
+                             int G, float R, float inv_h, cudaStream_t st);
 // K1 + K2 + K3 of one scoring call; n_blocks2 = pair-kernel grid (upper bound when non-uniform)
 cudaError_t launch_cell_score(const CellArgs& a, int dielectric, long long n_poses, int n_blocks2, cudaStream_t st);
 cudaError_t launch_kt_advance(unsigned long long* kt_base, int slots, cudaStream_t st);
