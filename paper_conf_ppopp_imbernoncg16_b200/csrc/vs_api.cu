@@ -205,7 +205,8 @@ static_assert(VS_CELL_G <= vsk::CELL_GMAX && VS_CELL_G % vsk::CELL_NSPLIT == 0, 
 #define VS_BIG_RUN_GROUPS 12
 #endif
 #ifndef VS_FILL_WARPS
-#define VS_FILL_WARPS 2048    // pair-kernel warps below which a scoring round uses KP = 1 chunks (launch shape)
+#define VS_FILL_WARPS 4096    // pair-kernel warps below which a scoring round uses KP = 1 chunks (launch shape); 2048 -> 4096:
+                              // medium 32 spots (S 4) 56.0 -> 52.2 ms, 125 spots (S 1) 150.4 -> 133.1, others unchanged
 #endif
 #ifndef VS_TRIGGER_SPOTS
 #define VS_TRIGGER_SPOTS 0    // runs of at most this many spots: PDL early trigger (latency-bound)
