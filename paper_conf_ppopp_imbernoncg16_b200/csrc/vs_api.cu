@@ -1155,6 +1155,10 @@ vs_status vs_create(const float* rec_xyz, const float* rec_q, const int32_t* rec
     CKT(pool::alloc(&sorted, sizeof(RecAtom) * std::max<int64_t>(tot, 1)), "alloc lists");
     c->cR = (float)reach + 0.01f;
     c->cell_g = cell_grid(c->nsplit);
+    if (const char* v = std::getenv("VS_CELL_GRID")) {  // tests / experiments: force the grid (speed only)
+      const int g = std::atoi(v);
+      if (g >= 4 && g <= CELL_GMAX && g % c->nsplit == 0) c->cell_g = g;
+    }
     const int G = c->cell_g;
     c->ch = 2.0f * c->cR / (float)G;
     c->cinv_h = (float)G / (2.0f * c->cR);

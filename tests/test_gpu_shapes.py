@@ -269,3 +269,35 @@ def test_run_stats_count_scored_poses_and_pairs(torch, preset, K):
     n_all = prob.cfg.n_spots
     assert st["poses_scored"] == per * (len(ids) + n_all)
     assert st["pairs"] == per * prob.cfg.n_lig * (int(sum(int(L[s]) for s in ids)) + int(sum(int(x) for x in L)))
+
+
+@pytest.mark.parametrize("S", [1, 4])
+def test_list_grid_changes_only_rounding(torch, oracle_mod, S):
+    """The per-spot list grid (cells per axis, a context property: 16 for 1-2 splits, 20 for 4; VS_CELL_GRID forces
+    it) decides which list atoms a chunk streams and their order inside a cell row, never which pairs contribute:
+    scores agree with the oracle at every grid, the within-rc census count is identical, and grids differ only by
+    fp32 summation order."""
+    prob = synth.make_problem("small")
+    spot, q, t = synth.make_poses(3000, prob.cfg.n_spots, 3.0, seed=23)
+    o = oracle_mod.Oracle.from_problem(prob, oracle_mod.score_params())
+    idx = np.arange(0, 3000, 10)
+    ref = o.score(spot[idx], q[idx], t[idx])
+    got, within = {}, {}
+    for G in (8, 12, 16, 20, 24):
+        old = os.environ.get("VS_CELL_GRID")
+        os.environ["VS_CELL_GRID"] = str(G)
+        try:
+            g = vs.Context.from_problem(prob, vs.score_params(list_splits=S))
+        finally:
+            if old is None:
+                os.environ.pop("VS_CELL_GRID", None)
+            else:
+                os.environ["VS_CELL_GRID"] = old
+        g.reset_stats()
+        g.set_timing(vs.TIMING_CENSUS)
+        got[G] = g.score_poses(spot, q, t)
+        within[G] = g.stats()["pairs_within"]
+        assert np.all(np.abs(got[G][idx] - ref) <= np.maximum(1e-4 * np.abs(ref), 1e-3)), G
+    assert len(set(within.values())) == 1, within
+    for G in got:
+        np.testing.assert_allclose(got[G], got[16], rtol=2e-6, atol=1e-4)
