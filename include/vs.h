@@ -182,7 +182,7 @@ VS_API vs_status vs_release_cached_memory(int32_t cuda_device);
  * order, and only VS_CELL_GRID changes that order):
  *   VS_GRAPHS=0             never capture CUDA graphs (plain launches, e.g. for profilers)
  *   VS_FILL_WARPS=n         scoring rounds with fewer pair-kernel warps than n use KP = 1 chunks (default 4096)
- *   VS_CELL_GRID=g          cells per axis of the per-spot list grid, 4..24, a multiple of list_splits (default 16
+ *   VS_CELL_GRID=g          cells per axis of the per-spot list grid, 4..24, a multiple of list_splits (default 18
  *                           for 1-2 list splits, 20 for 4; changes the list order inside a cell row, hence rounding)
  *   VS_SHAPE=1|2            force the chunk shape KP
  *   VS_DIRECT_GROUP_SPOTS=n spots per stream group at least in un-graphed runs (default 16)

@@ -183,17 +183,18 @@ struct DevBuf {
 #define VS_NSUB 12
 #endif
 constexpr int NSUB = VS_NSUB;  // spot groups (streams) of one vs_run
-// cells per axis of the per-spot list grid: 16 for contexts with 1 or 2 list splits (throughput-bound runs: fewer,
+// cells per axis of the per-spot list grid: 18 for contexts with 1 or 2 list splits (throughput-bound runs: fewer,
 // longer row runs), 20 with 4 splits (latency-bound runs: each split warp streams fewer atoms).  Medium, ms: S 1,
-// 500 spots: G 24 / 20 / 16 / 12 465.3 / 464.2 / 459.9 / 462.4; S 2, 125 spots 129.0 / 128.1 / 127.3; S 4, 63
-// spots 78.0 / 77.1 / 78.5; small (S 4) 17.9 / 17.57 / 18.2; large 500 spots (S 1) 1260 / 1256 / 1247
-// (profiles/r02_notes.md).  S must divide G (the pair kernel assigns cell rows to splits by cy mod S).
+// 500 spots: G 24 / 20 / 18 / 16 / 14 / 12 465.3 / 464.2 / 458.9 / 460.3 / 460.1 / 462.4; S 2, 125 spots G 24 / 20 /
+// 18 / 16 / 14: 129.0 / 128.1 / 127.0 / 127.4 / 133.5; S 4, 63 spots G 24 / 20 / 16: 78.0 / 77.1 / 78.5; small (S 4)
+// 17.9 / 17.57 / 18.2; large 500 spots (S 1) G 24 / 20 / 18 / 16: 1260 / 1256 / 1248 / 1250 (profiles/r02_notes.md).
+// S must divide G (the pair kernel assigns cell rows to splits by cy mod S).
 int cell_grid(int nsplit) {
-  const int g = VS_CELL_G > 0 ? VS_CELL_G : (nsplit >= 4 ? 20 : 16);
+  const int g = VS_CELL_G > 0 ? VS_CELL_G : (nsplit >= 4 ? 20 : 18);
   return g;
 }
-static_assert(vsk::CELL_GMAX % vsk::CELL_NSPLIT == 0 && 20 % vsk::CELL_NSPLIT == 0 && 16 % vsk::CELL_NSPLIT == 0,
-              "the pair kernel assigns cell rows to splits by cy mod S");
+static_assert(vsk::CELL_GMAX % vsk::CELL_NSPLIT == 0 && 20 % vsk::CELL_NSPLIT == 0 && 18 % 2 == 0,
+              "the pair kernel assigns cell rows to splits by cy mod S (18: 1 or 2 splits, 20: 4)");
 static_assert(VS_CELL_G <= vsk::CELL_GMAX && VS_CELL_G % vsk::CELL_NSPLIT == 0, "VS_CELL_G");
 #ifndef VS_GROUP_SPOTS
 #define VS_GROUP_SPOTS 8    // spots per stream group at least
@@ -252,7 +253,7 @@ struct vs_ctx {
   unsigned long long host_poses = 0, host_pairs = 0;
   uint64_t* d_seed = nullptr;           // seed of the current run (device copy)
   uint16_t* d_cells = nullptr;          // cutoff mode: [n_spots][cg^3 + 1] cell starts of the cell-sorted lists
-  int cell_g = 16;                      // cells per axis of the list grid (cell_grid)
+  int cell_g = 18;                      // cells per axis of the list grid (cell_grid)
   float cR = 0.0f, ch = 0.0f, cinv_h = 0.0f;
   long long fill_warps = VS_FILL_WARPS;  // launch shape target (speed only)
   int nsplit = 1;                        // canonical receptor-list splits (vs_score_params.list_splits)

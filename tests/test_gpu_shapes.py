@@ -273,7 +273,7 @@ def test_run_stats_count_scored_poses_and_pairs(torch, preset, K):
 
 @pytest.mark.parametrize("S", [1, 4])
 def test_list_grid_changes_only_rounding(torch, oracle_mod, S):
-    """The per-spot list grid (cells per axis, a context property: 16 for 1-2 splits, 20 for 4; VS_CELL_GRID forces
+    """The per-spot list grid (cells per axis, a context property: 18 for 1-2 splits, 20 for 4; VS_CELL_GRID forces
     it) decides which list atoms a chunk streams and their order inside a cell row, never which pairs contribute:
     scores agree with the oracle at every grid, the within-rc census count is identical, and grids differ only by
     fp32 summation order."""
