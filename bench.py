@@ -110,6 +110,12 @@ class ClockSampler:
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            # nvidia-smi takes a few hundred ms to start sampling: wait for its first line, so that a short timed
+            # region (small config) is sampled too
+            t0 = time.perf_counter()
+            while not self.lines and time.perf_counter() - t0 < 3.0 and self.proc.poll() is None:
+                time.sleep(0.01)
+            self.lines.clear()
         except OSError:
             self.proc = None
 
@@ -126,6 +132,13 @@ class ClockSampler:
         except subprocess.TimeoutExpired:
             self.proc.kill()
         self.t.join(timeout=2)
+        if not self.lines:  # a region shorter than the 100 ms period: one query right after it
+            try:
+                r = subprocess.run(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                    "-i", str(self.idx)], capture_output=True, text=True, timeout=20)
+                self.lines = [x.strip() for x in r.stdout.splitlines() if x.strip()]
+            except (OSError, subprocess.SubprocessError):
+                pass
         sm, mx, reasons = [], 0.0, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in self.lines:
@@ -520,10 +533,10 @@ def main():
     for c in work_ctx:
         c.reset_stats()
     clocks = ClockSampler(local, enabled=(rank == 0 and not args.no_clocks))
+    clocks.start()   # before the barrier: the sampler is running when every rank enters the timed region
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize(dev)
-    clocks.start()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(main_stream)
     for i in range(args.steps):
